@@ -1,0 +1,133 @@
+/*
+ * tbs.h — C ABI of the B200-native 2-body-statistics (2-BS) library, libtbs.so.
+ *
+ * The operations are the three output types of Pitaksirianan, Nouri & Tu,
+ * "Efficient 2-Body Statistics Computation on GPUs" (ICPP 2016). Citations are to
+ * /root/reference/PAPER.md lines (L<a>-<b>) with the section they fall in.
+ *
+ *   2-BS (§I): a statistic over all pairs of an N-point set computed from a
+ *   pairwise "distance function". Every unordered pair {i, j}, i != j, contributes
+ *   exactly once (Alg. 1 loops i = t+1..N, L290-296; Alg. 2).
+ *   Distance = Euclidean (L600-602, L841-843).
+ *
+ *   tbs_sdh        Type-II output (§III-B, §IV-D): the spatial
+ *                  distance histogram, hist[k] = #{i<j : min(floor(d_ij / w), nb-1) = k}.
+ *   tbs_pcf        Type-I output (§III-B, §IV-B): the 2-point
+ *                  correlation count, #{i<j : d_ij < r}.
+ *   tbs_pairmatrix Type-III output (§III-B, §IV-C): the full pairwise
+ *                  kernel matrix out[i][j] = K(p_i, p_j), diagonal included.
+ *
+ * Readings of points the paper leaves open are listed in DESIGN.md §Readings
+ * (half-open buckets, clamping of d >= nb*w into the last bucket, d < r for 2PCF,
+ * Gaussian kernel for Type-III).
+ *
+ * ---- Memory and ownership --------------------------------------------------------
+ * points   AoS float32 [n][dim], row-major, read-only, caller-owned.
+ * hist     uint64 [nbuckets], caller-allocated, OVERWRITTEN (not accumulated).
+ * count    uint64 [1], caller-allocated, overwritten.
+ * out      float32 [row_end - row_begin][n] row-major, caller-allocated, overwritten.
+ * The simple entry points (tbs_sdh, tbs_pcf, tbs_pairmatrix) accept HOST or DEVICE
+ * pointers (detected with cudaPointerGetAttributes; all arrays of one call must be
+ * on the same side), run on a library stream and return after the result is in
+ * place (synchronous). The _ex entry points take DEVICE pointers only, enqueue on
+ * args->stream and return without synchronising: results are valid once that
+ * stream has been synchronised. Scratch (the SoA coordinate copy, partial
+ * histograms) is allocated stream-ordered from the device's default memory pool
+ * and returned to it at the end of each call; tbs_release() trims the pool.
+ *
+ * ---- Errors ------------------------------------------------------------------------
+ * Every function returns a tbs_status. Argument errors are detected synchronously,
+ * return TBS_EINVAL and enqueue nothing: n < 0 or n > TBS_MAX_N; dim outside [1,4];
+ * nbuckets < 1 or > TBS_MAX_BUCKETS; bucket_width <= 0 or non-finite; radius < 0 or
+ * NaN; NULL array with n >= 2 (or a NULL output); a row range outside [0, n];
+ * TBS_EXACT_LATTICE with a bucket width that is not m * 2^-j (m, j integers,
+ * 1 <= m < 2^20, 0 <= j <= 20). n < 2 (or an empty row range) is valid and yields
+ * zero output. Allocation failure returns TBS_ENOMEM; a CUDA error returns
+ * TBS_ECUDA. tbs_last_error() gives a thread-local message for the last non-OK
+ * status. Non-finite coordinates are a caller contract violation (not checked on
+ * the hot path). Under TBS_EXACT_LATTICE, coordinates must be integer-valued with
+ * every squared pair distance < 2^24 (exact in fp32) and 4^j * s < 2^62.
+ */
+#ifndef TBS_H_
+#define TBS_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  TBS_OK = 0,
+  TBS_EINVAL = 1,
+  TBS_ENOMEM = 2,
+  TBS_ECUDA = 3,
+  TBS_EUNSUPPORTED = 4
+} tbs_status;
+
+/* Type-III pair functions. TBS_K_GAUSSIAN is exp(-gamma * ||x - y||^2) (reading Q10). */
+typedef enum { TBS_K_GAUSSIAN = 0, TBS_K_DIST2 = 1, TBS_K_DIST = 2 } tbs_kernel_type;
+typedef struct {
+  int type;     /* tbs_kernel_type */
+  float gamma;  /* TBS_K_GAUSSIAN only */
+} tbs_kernel;
+
+/* Flags for tbs_args.flags. */
+#define TBS_EXACT_LATTICE 0x1u        /* SDH: exact integer squared-distance bucketing   */
+#define TBS_HIST_FORCE_LANE 0x10u     /* SDH: 32 lane-private smem copies per CTA          */
+#define TBS_HIST_FORCE_CTA 0x20u      /* SDH: one shared smem copy per CTA                 */
+#define TBS_HIST_FORCE_GLOBAL 0x40u   /* SDH: partially privatised global u64 copies       */
+#define TBS_FORCE_CLAMP 0x100u        /* SDH: never elide the nb-1 clamp (ablation/tests)   */
+
+#define TBS_MAX_N ((int64_t)1 << 30)
+#define TBS_MAX_BUCKETS (1 << 24)
+
+/* ---- simple entry points (north-star signatures), host or device pointers -------- */
+
+/* SDH over all pairs of points[n][dim]: hist[k] = #{i<j : min(floor(d/w), nb-1) = k}. */
+int tbs_sdh(const float* points, int64_t n, int dim, float bucket_width, int nbuckets, uint64_t* hist);
+
+/* 2PCF over all pairs of points[n][3]: *count = #{i<j : d < radius}. */
+int tbs_pcf(const float* points, int64_t n, float radius, uint64_t* count);
+
+/* Type-III over points[n][3]: out[i*n + j] = K(p_i, p_j) for all i, j in [0, n). */
+int tbs_pairmatrix(const float* points, int64_t n, tbs_kernel kernel, float* out);
+
+/* ---- extended entry points: device pointers, caller stream, row ranges ------------- */
+typedef struct {
+  const float* points;  /* device AoS float32 [n][dim]                                     */
+  int64_t n;
+  int dim;              /* 1..4                                                            */
+  int64_t row_begin;    /* anchors i in [row_begin, row_end) pair with every j > i          */
+  int64_t row_end;      /* (Type-III: rows i in [row_begin,row_end) against all j in [0,n)) */
+  void* stream;         /* cudaStream_t; NULL = legacy default stream                      */
+  uint32_t flags;       /* TBS_* flags above                                               */
+  void* ev_begin;       /* optional cudaEvent_t recorded just before the pair kernel        */
+  void* ev_end;         /* optional cudaEvent_t recorded just after it (profiling hook)     */
+} tbs_args;
+
+int tbs_sdh_ex(const tbs_args* args, float bucket_width, int nbuckets, uint64_t* hist);
+int tbs_pcf_ex(const tbs_args* args, float radius, uint64_t* count);
+int tbs_pairmatrix_ex(const tbs_args* args, tbs_kernel kernel, float* out);
+
+/* Pair-count-balanced anchor-row partition for multi-GPU: rank r of
+ * `world` gets [*row_begin, *row_end) such that sum over its rows of (n-1-i) is
+ * n(n-1)/(2*world) up to one row; the ranges are disjoint and cover [0, n). Host-only. */
+int tbs_rank_rows(int64_t n, int world, int rank, int64_t* row_begin, int64_t* row_end);
+
+/* Thread-local text of the last non-OK status ("" if none). */
+const char* tbs_last_error(void);
+
+/* Trim the cached scratch of the current device's default memory pool. */
+void tbs_release(void);
+
+/* Number of kernels this library has launched in this process (evidence counter). */
+uint64_t tbs_launch_count(void);
+
+/* ABI version (major * 100 + minor). */
+int tbs_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TBS_H_ */

@@ -1,0 +1,146 @@
+"""CPU oracle for the 2-BS hot path — TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
+and ``--impl reference`` legs may import this package. The product package
+(``paper_conf_icpp_pitaksirianannt16_b200``) never imports it and shares no code
+with it. The arithmetic lives in ``tbs_oracle.c`` (plain C + OpenMP, double
+precision); this file only marshals numpy arrays through ctypes.
+
+Functions and their pins (tests/test_oracle_pins.py):
+  sdh            brute force (numpy pdist-style), mass, hand cases, cube closed form
+  sdh_lattice    hand cases (edge ties), brute force, closed form lattice_closed
+  pcf            brute force, cumulative-SDH identity, cube closed form
+  pairmatrix     torch.cdist float64 (library routine), symmetry, diagonal
+  lattice_closed brute force of sdh_lattice on permuted lattices
+Parity status: no worked example in PAPER.md prints values, so every pin is a
+mathematical one; see DESIGN.md §Oracle.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "tbs_oracle.c")
+_LIB = os.path.join(_HERE, "libtbs_oracle.so")
+_lib = None
+
+_u64p = ctypes.POINTER(ctypes.c_uint64)
+_f32p = ctypes.POINTER(ctypes.c_float)
+_f64p = ctypes.POINTER(ctypes.c_double)
+_i64 = ctypes.c_int64
+
+
+def build(force: bool = False) -> str:
+    """Compile the oracle with gcc (-O2 -ffp-contract=off -fopenmp)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fopenmp", "-fPIC", "-shared",
+                               "-std=c11", "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        build()
+        lib = ctypes.CDLL(_LIB)
+        lib.oracle_sdh.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, ctypes.c_int, _i64, _i64,
+                                   _u64p, _u64p]
+        lib.oracle_sdh_lattice.argtypes = [_f32p, _i64, ctypes.c_int, _i64, ctypes.c_int, ctypes.c_int,
+                                           _i64, _i64, _u64p]
+        lib.oracle_pcf.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, _i64, _i64, _u64p, _u64p]
+        lib.oracle_pairmatrix.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, _i64, _i64, _f64p]
+        lib.oracle_lattice_closed.argtypes = [_i64, _i64, ctypes.c_int, ctypes.c_int, _u64p, _i64, _u64p]
+        lib.oracle_num_threads.restype = ctypes.c_int
+        _lib = lib
+    return _lib
+
+
+def _pts(points):
+    p = np.ascontiguousarray(points, dtype=np.float32)
+    if p.ndim == 1:
+        p = p.reshape(-1, 1)
+    return p, p.shape[0], p.shape[1]
+
+
+def _ptr(a, t):
+    return a.ctypes.data_as(t)
+
+
+def _rows(rows, n):
+    return (0, n) if rows is None else (int(rows[0]), int(rows[1]))
+
+
+def num_threads() -> int:
+    return _load().oracle_num_threads()
+
+
+def sdh(points, bucket_width, nbuckets, rows=None, with_amb=True):
+    """Float-mode SDH. ``bucket_width`` is rounded to fp32 first (the API's type).
+
+    Returns (hist uint64[nb], amb uint64[nb+1]) — amb[e] counts pairs within 1e-6
+    relative of edge e (e = 1..nb-1).
+    """
+    p, n, dim = _pts(points)
+    rb, re = _rows(rows, n)
+    hist = np.zeros(nbuckets, np.uint64)
+    amb = np.zeros(nbuckets + 1, np.uint64)
+    w = float(np.float32(bucket_width))
+    rc = _load().oracle_sdh(_ptr(p, _f32p), n, dim, w, int(nbuckets), rb, re, _ptr(hist, _u64p),
+                            _ptr(amb, _u64p) if with_amb else None)
+    if rc:
+        raise ValueError(f"oracle_sdh: status {rc}")
+    return hist, amb
+
+
+def sdh_lattice(points, m, j, nbuckets, rows=None):
+    """Exact-lattice SDH, bucket width w = m * 2^-j (integer-valued coordinates)."""
+    p, n, dim = _pts(points)
+    rb, re = _rows(rows, n)
+    hist = np.zeros(nbuckets, np.uint64)
+    rc = _load().oracle_sdh_lattice(_ptr(p, _f32p), n, dim, int(m), int(j), int(nbuckets), rb, re,
+                                    _ptr(hist, _u64p))
+    if rc:
+        raise ValueError(f"oracle_sdh_lattice: status {rc}")
+    return hist
+
+
+def pcf(points, radius, rows=None):
+    """2PCF count #{i<j : d < r} and its ambiguity count (|d - r| <= 1e-6 r)."""
+    p, n, dim = _pts(points)
+    rb, re = _rows(rows, n)
+    c = np.zeros(1, np.uint64)
+    a = np.zeros(1, np.uint64)
+    rc = _load().oracle_pcf(_ptr(p, _f32p), n, dim, float(np.float32(radius)), rb, re, _ptr(c, _u64p),
+                            _ptr(a, _u64p))
+    if rc:
+        raise ValueError(f"oracle_pcf: status {rc}")
+    return int(c[0]), int(a[0])
+
+
+def pairmatrix(points, gamma, rows=None):
+    """Gaussian pair matrix rows [rb, re) x n in float64."""
+    p, n, dim = _pts(points)
+    rb, re = _rows(rows, n)
+    out = np.zeros((re - rb, n), np.float64)
+    rc = _load().oracle_pairmatrix(_ptr(p, _f32p), n, dim, float(np.float32(gamma)), rb, re,
+                                   _ptr(out, _f64p))
+    if rc:
+        raise ValueError(f"oracle_pairmatrix: status {rc}")
+    return out
+
+
+def lattice_closed(L, m, j, nbuckets, r2=-1):
+    """Closed-form lattice SDH of {0..L-1}^3 (and 2PCF count s < r2 if r2 >= 0)."""
+    hist = np.zeros(nbuckets, np.uint64)
+    c = np.zeros(1, np.uint64)
+    rc = _load().oracle_lattice_closed(int(L), int(m), int(j), int(nbuckets), _ptr(hist, _u64p), int(r2),
+                                       _ptr(c, _u64p))
+    if rc:
+        raise ValueError(f"oracle_lattice_closed: status {rc}")
+    return hist, int(c[0])

@@ -1,0 +1,264 @@
+"""Pins for the CPU oracle (oracle/), independent of the oracle's own code.
+
+PAPER.md prints no worked example with values, so every pin is a
+mathematical one: hand cases, brute force with independent numpy/scipy/torch
+routines, mass, exact lattice closed forms, the uniform-cube distance law, and
+cross-API identities. Each test names the passage it follows.
+"""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+from scipy.spatial.distance import pdist
+
+import oracle
+import tbs_inputs as g
+import cube_cdf  # tests/cube_cdf.py (sibling helper)
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def brute_sdh(p, w, nb):
+    """Independent SDH: scipy pdist (i<j pairs, L290-296) -> floor(d/w) clamped (Q1, Q2)."""
+    d = pdist(p.astype(np.float64))
+    q = d / np.float64(np.float32(w))
+    b = np.minimum(np.floor(q), nb - 1).astype(np.int64)
+    return np.bincount(b, minlength=nb).astype(np.uint64), d
+
+
+def brute_lattice(p, m, j, nb):
+    """Independent exact lattice bucketing with python integers (math.isqrt)."""
+    pi = p.astype(np.int64)
+    n = len(pi)
+    h = np.zeros(nb, np.uint64)
+    for i in range(n):
+        s = ((pi[i + 1:] - pi[i]) ** 2).sum(axis=1)
+        for sv in s.tolist():
+            k = min(math.isqrt(sv << (2 * j)) // m, nb - 1)
+            h[k] += 1
+    return h
+
+
+# ---------------------------------------------------------------- hand cases (golden)
+def test_hand_cases_golden():
+    """tests/golden/hand_cases.json: values derived by hand (see its 'why' fields)."""
+    with open(os.path.join(GOLDEN, "hand_cases.json")) as f:
+        cases = json.load(f)["cases"]
+    for c in cases:
+        p = np.array(c["points"], np.float32).reshape(-1, 3)
+        if c["op"] == "sdh":
+            h, _ = oracle.sdh(p, c["w"], c["nb"])
+            assert h.tolist() == c["hist"], c["why"]
+        elif c["op"] == "sdh_lattice":
+            h = oracle.sdh_lattice(p, c["m"], c["j"], c["nb"])
+            assert h.tolist() == c["hist"], c["why"]
+        elif c["op"] == "pcf":
+            cnt, _ = oracle.pcf(p, c["r"])
+            assert cnt == c["count"], c["why"]
+        elif c["op"] == "pairmatrix":
+            out = oracle.pairmatrix(p, c["gamma"])
+            np.testing.assert_allclose(out, np.array(c["out"]), rtol=1e-15, err_msg=c["why"])
+
+
+@pytest.mark.parametrize("n", [0, 1])
+def test_degenerate_sizes(n):
+    p = g.uniform(n, 1)
+    h, a = oracle.sdh(p, 0.1, 16)
+    assert h.sum() == 0 and a.sum() == 0
+    assert oracle.pcf(p, 0.5)[0] == 0
+
+
+def test_all_coincident():
+    p = np.full((300, 3), 0.25, np.float32)
+    h, a = oracle.sdh(p, 0.01, 10)
+    assert h[0] == 300 * 299 // 2 and h[1:].sum() == 0
+    assert oracle.pcf(p, 1e-3)[0] == 300 * 299 // 2
+    assert oracle.pcf(p, 0.0)[0] == 0          # d < 0 never (reading Q4: strict)
+
+
+# ---------------------------------------------------------------- brute force
+@pytest.mark.parametrize("kind,n,nb,seed", [("uniform", 1500, 64, 11), ("uniform", 777, 7, 12),
+                                            ("clustered", 1800, 256, 13)])
+def test_sdh_bruteforce(kind, n, nb, seed):
+    p = g.make(kind, n, seed)
+    w = float(np.float32(math.sqrt(3) / nb))
+    h, amb = oracle.sdh(p, w, nb)
+    hb, d = brute_sdh(p, w, nb)
+    assert h.tolist() == hb.tolist()
+    # ambiguity counts: |d - e w| <= 1e-6 e w for e = 1..nb-1
+    wd = np.float64(np.float32(w))
+    e = np.rint(d / wd)
+    ok = (e >= 1) & (e <= nb - 1) & (np.abs(d - e * wd) <= 1e-6 * e * wd)
+    ab = np.bincount(e[ok].astype(np.int64), minlength=nb + 1)
+    assert amb.tolist() == ab.tolist()
+
+
+def test_sdh_dims_1_2_4():
+    for dim in (1, 2, 4):
+        p = g.uniform(600, 21 + dim, dim)
+        w = float(np.float32(math.sqrt(dim) / 32))
+        h, _ = oracle.sdh(p, w, 32)
+        hb, _ = brute_sdh(p, w, 32)
+        assert h.tolist() == hb.tolist()
+
+
+def test_mass_invariant_4096():
+    """Sum of the histogram = n(n-1)/2 exactly (each unordered pair once, L290-296)."""
+    p = g.uniform(4096, 1)
+    h, _ = oracle.sdh(p, float(np.float32(math.sqrt(3) / 64)), 64)
+    assert int(h.sum()) == 4096 * 4095 // 2 == 8386560
+
+
+def test_pcf_bruteforce():
+    p = g.clustered(2000, 3)
+    for r in (0.0, 0.005, 0.03, 0.3, 2.0):
+        c, a = oracle.pcf(p, r)
+        d = pdist(p.astype(np.float64))
+        rr = np.float64(np.float32(r))
+        assert c == int((d < rr).sum())
+        assert a == int((np.abs(d - rr) <= 1e-6 * rr).sum())
+
+
+def test_pcf_equals_cumulative_sdh_on_lattice():
+    """2PCF(r = e w) == sum_{b<e} SDH[b] (reading Q4), exact on lattices."""
+    p = g.lattice(9, 5)
+    h = oracle.sdh_lattice(p, 1, 0, 20)
+    for e in range(1, 20):
+        c, _ = oracle.pcf(p, float(e))
+        assert c == int(h[:e].sum())
+
+
+# ---------------------------------------------------------------- rows
+def test_row_ranges_partition():
+    p = g.uniform(1000, 7)
+    w = float(np.float32(0.02))
+    full, famb = oracle.sdh(p, w, 100)
+    cuts = [0, 1, 170, 171, 500, 999, 1000]
+    acc = np.zeros(100, np.uint64)
+    accc = 0
+    for a, b in zip(cuts[:-1], cuts[1:]):
+        acc += oracle.sdh(p, w, 100, rows=(a, b))[0]
+        accc += oracle.pcf(p, 0.1, rows=(a, b))[0]
+    assert acc.tolist() == full.tolist()
+    assert accc == oracle.pcf(p, 0.1)[0]
+
+
+def test_row_range_is_anchor_subset():
+    """rows [a,b): anchors i in [a,b) with all partners j>i."""
+    p = g.uniform(400, 8)
+    d = np.sqrt(((p[:, None, :].astype(np.float64) - p[None, :, :]) ** 2).sum(-1))
+    i, j = np.triu_indices(400, 1)
+    sel = (i >= 100) & (i < 250)
+    w = np.float64(np.float32(0.05))
+    b = np.minimum(np.floor(d[i[sel], j[sel]] / w), 39).astype(np.int64)
+    h, _ = oracle.sdh(p, 0.05, 40, rows=(100, 250))
+    assert h.tolist() == np.bincount(b, minlength=40).tolist()
+
+
+# ---------------------------------------------------------------- lattice exact mode
+@pytest.mark.parametrize("L,m,j,nb", [(6, 2, 0, 6), (7, 1, 1, 8), (7, 3, 1, 12), (5, 1, 0, 3), (6, 5, 3, 40)])
+def test_lattice_oracle_vs_bruteforce(L, m, j, nb):
+    p = g.lattice(L, 100 + L)
+    h = oracle.sdh_lattice(p, m, j, nb)
+    assert h.tolist() == brute_lattice(p, m, j, nb).tolist()
+    assert int(h.sum()) == len(p) * (len(p) - 1) // 2
+
+
+@pytest.mark.parametrize("L,m,j,nb", [(6, 2, 0, 6), (7, 1, 1, 8), (7, 3, 1, 12), (5, 1, 0, 3), (8, 1, 2, 50)])
+def test_lattice_closed_form_vs_bruteforce(L, m, j, nb):
+    """O(L^3) closed form == brute force on a permuted lattice (any point order)."""
+    p = g.lattice(L, 7)
+    hc, _ = oracle.lattice_closed(L, m, j, nb)
+    assert hc.tolist() == brute_lattice(p, m, j, nb).tolist()
+
+
+def test_lattice_closed_known_values():
+    """Values recomputed independently in SURVEY Appendix A item 4."""
+    assert oracle.lattice_closed(6, 2, 0, 6)[0].tolist() == [1940, 9472, 10068, 1712, 28, 0]
+    assert oracle.lattice_closed(7, 1, 1, 8)[0].tolist() == [0, 0, 2394, 864, 5415, 1050, 6632, 42298]
+
+
+def test_lattice_closed_pcf():
+    """Closed-form lattice 2PCF (s < r^2) == brute force == oracle.pcf at r = 4 (r^2 = 16)."""
+    p = g.lattice(8, 3)
+    _, c = oracle.lattice_closed(8, 1, 0, 4, r2=16)
+    d2 = pdist(p.astype(np.float64), "sqeuclidean")
+    assert c == int((d2 < 16).sum()) == oracle.pcf(p, 4.0)[0]
+
+
+def test_float_mode_equals_lattice_mode_on_dyadic_width():
+    """On integer points with a dyadic width, floor(d/w) in double is exact."""
+    p = g.lattice(9, 2)
+    for (m, j) in [(1, 0), (3, 2), (1, 3)]:
+        w = m * 2.0 ** -j
+        hf, _ = oracle.sdh(p, w, 64)
+        hl = oracle.sdh_lattice(p, m, j, 64)
+        assert hf.tolist() == hl.tolist()
+
+
+def test_lattice_rejects_non_integer():
+    with pytest.raises(ValueError):
+        oracle.sdh_lattice(np.array([[0.5, 0, 0], [1, 1, 1]], np.float32), 1, 0, 4)
+
+
+# ---------------------------------------------------------------- uniform cube law
+def test_cube_cdf_quadrature_pins():
+    for r in (0.1, 0.5, 0.9, 1.0):
+        assert abs(cube_cdf.F(r) - cube_cdf.F_closed_le1(r)) < 1e-9
+    assert cube_cdf.F(math.sqrt(3)) == 1.0
+    # mean distance = int_0^sqrt3 (1 - F) dr = Robbins' constant
+    from scipy import integrate
+    mean, _ = integrate.quad(lambda r: 1 - cube_cdf.F(r), 0, math.sqrt(3), points=[1, math.sqrt(2)], limit=200)
+    assert abs(mean - cube_cdf.ROBBINS) < 1e-7
+
+
+def test_sdh_uniform_matches_cube_law():
+    """E[h_k] = C(n,2) (F(r_{k+1}) - F(r_k)); tolerance 6 sigma with the U-statistic
+    variance C(n,2) p(1-p) + n(n-1)(n-2) zeta_1 (pairs sharing a point correlate)."""
+    n, nb = 4096, 64
+    w = float(np.float32(math.sqrt(3) / nb))
+    p = g.uniform(n, 1)
+    h, _ = oracle.sdh(p, w, nb)
+    edges = [cube_cdf.F(k * np.float64(np.float32(w))) for k in range(nb)] + [1.0]
+    pk = np.diff(np.array(edges))
+    npairs = n * (n - 1) // 2
+    # zeta_1 estimated from per-point row histograms (independent numpy computation)
+    x = p.astype(np.float64)
+    zeta = np.zeros(nb)
+    cnt = np.zeros((n, nb))
+    for i in range(0, n, 512):
+        d = np.sqrt(((x[i:i + 512, None, :] - x[None, :, :]) ** 2).sum(-1))
+        b = np.minimum(np.floor(d / np.float64(np.float32(w))), nb - 1).astype(np.int64)
+        for r in range(b.shape[0]):
+            row = np.bincount(b[r], minlength=nb).astype(np.float64)
+            row[0] -= 1                      # self pair
+            cnt[i + r] = row
+    zeta = (cnt / (n - 1)).var(axis=0)
+    var = npairs * pk * (1 - pk) + n * (n - 1) * (n - 2) * zeta
+    dev = np.abs(h.astype(np.float64) - npairs * pk)
+    assert np.all(dev <= 6 * np.sqrt(var) + 1), (dev / np.sqrt(var + 1e-12)).max()
+
+
+# ---------------------------------------------------------------- Type-III
+def test_pairmatrix_vs_cdist():
+    import torch
+    p = g.uniform(700, 4)
+    gamma = 1.0
+    out = oracle.pairmatrix(p, gamma)
+    t = torch.from_numpy(p.astype(np.float64))
+    d = torch.cdist(t, t, compute_mode="donot_use_mm_for_euclid_dist")
+    ref = torch.exp(-gamma * d * d).numpy()
+    np.testing.assert_allclose(out, ref, rtol=1e-13, atol=0)
+    assert np.array_equal(out, out.T)
+    assert np.all(np.diag(out) == 1.0)
+    rows = oracle.pairmatrix(p, gamma, rows=(100, 140))
+    assert np.array_equal(rows, out[100:140])
+
+
+def test_pairmatrix_lattice_values():
+    p = g.lattice(4, 1)
+    out = oracle.pairmatrix(p, 0.5)
+    s = ((p[:, None, :].astype(np.int64) - p[None, :, :]) ** 2).sum(-1)
+    np.testing.assert_allclose(out, np.exp(-0.5 * s.astype(np.float64)), rtol=1e-15, atol=0)

@@ -1,0 +1,191 @@
+// Microbenchmarks for the pipe peaks that bound the 2-BS hot path on sm_100a
+// (SURVEY.md §8(d) "Microbenchmarks that define the peaks").
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o tools/peaks tools/peaks.cu
+// Prints one JSON object: per-op lane-ops/s, lane-ops/clk/SM, and the SM clock seen.
+#include <cstdio>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#define CK(x) do { cudaError_t e_ = (x); if (e_ != cudaSuccess) { \
+  fprintf(stderr, "%s:%d %s\n", __FILE__, __LINE__, cudaGetErrorString(e_)); return 1; } } while (0)
+
+constexpr int ITERS = 4096;
+
+// ---- clock probe: SM cycles vs ns over a busy loop -------------------------
+__global__ void k_clock(unsigned long long* out, int spin) {
+  unsigned long long c0 = clock64(), t0, t1;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  float x = threadIdx.x;
+  for (int i = 0; i < spin; ++i) x = fmaf(x, 0.999f, 0.5f);
+  unsigned long long c1 = clock64();
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+  if (threadIdx.x == 0) { out[2 * blockIdx.x] = c1 - c0; out[2 * blockIdx.x + 1] = t1 - t0; }
+  if (x == -1.f) out[0] = 0;
+}
+
+// ---- FP32 scalar FFMA, all-register operands ------------------------------
+__global__ void k_ffma(float* out, float y0, float z0) {
+  float y = y0 + threadIdx.x * 1e-9f, z = z0 - threadIdx.x * 1e-9f;
+  float x[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) x[c] = threadIdx.x + c;
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) x[c] = fmaf(x[c], y, z);
+  }
+  float s = 0; for (int c = 0; c < 8; ++c) s += x[c];
+  if (s == 1.2345f) out[0] = s;
+}
+
+// ---- FP32 packed FFMA2 (fma.rn.f32x2) ---------------------------------------
+__global__ void k_ffma2(float* out, float y0, float z0) {
+  float2 y = make_float2(y0 + threadIdx.x * 1e-9f, y0), z = make_float2(z0, z0 - threadIdx.x * 1e-9f);
+  float2 x[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) x[c] = make_float2(threadIdx.x + c, c);
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) x[c] = __ffma2_rn(x[c], y, z);
+  }
+  float s = 0; for (int c = 0; c < 8; ++c) s += x[c].x + x[c].y;
+  if (s == 1.2345f) out[0] = s;
+}
+
+// ---- FP32 scalar FADD / packed FADD2 ----------------------------------------
+__global__ void k_fadd(float* out, float y0) {
+  float y = y0 + threadIdx.x * 1e-9f;
+  float x[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) x[c] = threadIdx.x + c;
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) x[c] = x[c] - y;
+  }
+  float s = 0; for (int c = 0; c < 8; ++c) s += x[c];
+  if (s == 1.2345f) out[0] = s;
+}
+__global__ void k_fadd2(float* out, float y0) {
+  float2 y = make_float2(y0 + threadIdx.x * 1e-9f, y0);
+  float2 x[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) x[c] = make_float2(threadIdx.x + c, c);
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) x[c] = __fadd2_rn(x[c], y);
+  }
+  float s = 0; for (int c = 0; c < 8; ++c) s += x[c].x + x[c].y;
+  if (s == 1.2345f) out[0] = s;
+}
+
+// ---- MUFU: sqrt.approx / rsqrt.approx / ex2.approx ---------------------------
+template <int OP>
+__global__ void k_mufu(float* out) {
+  float x[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) x[c] = 1.5f + threadIdx.x * 1e-3f + c;
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      if (OP == 0) asm volatile("sqrt.approx.f32 %0, %0;" : "+f"(x[c]));
+      if (OP == 1) asm volatile("rsqrt.approx.f32 %0, %0;" : "+f"(x[c]));
+      if (OP == 2) asm volatile("ex2.approx.f32 %0, %0;" : "+f"(x[c]));
+    }
+  }
+  float s = 0; for (int c = 0; c < 8; ++c) s += x[c];
+  if (s == 1.2345f) out[0] = s;
+}
+
+// ---- shared-memory atomics ---------------------------------------------------
+// MODE 0: lane-private rows (word 32*k + lane): no bank conflict, no same address.
+// MODE 1: one copy of 256 bins, pseudo-random bin per lane (random bank conflicts).
+// MODE 2: all lanes of a warp hit one address.
+template <int MODE>
+__global__ void k_atoms(unsigned* out) {
+  extern __shared__ unsigned h[];
+  const int lane = threadIdx.x & 31;
+  for (int i = threadIdx.x; i < 64 * 32; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  unsigned k[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) k[c] = (threadIdx.x * 2654435761u) ^ (c * 40503u);
+  unsigned* base = h + lane;
+  for (int i = 0; i < ITERS / 4; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      k[c] = k[c] * 1664525u + 1013904223u;
+      if (MODE == 0) atomicAdd(base + ((k[c] >> 26) << 5), 1u);
+      if (MODE == 1) atomicAdd(h + (k[c] >> 24), 1u);
+      if (MODE == 2) atomicAdd(h + (c << 5), 1u);
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0 && h[5] == 0xffffffffu) out[0] = h[0];
+}
+
+// ---- LDS.128 broadcast ---------------------------------------------------------
+__global__ void k_lds128(float* out) {
+  __shared__ float4 s[1024];
+  for (int i = threadIdx.x; i < 1024; i += blockDim.x) s[i] = make_float4(i, i + 1, i + 2, i + 3);
+  __syncthreads();
+  float4 a = make_float4(0, 0, 0, 0);
+  for (int i = 0; i < ITERS; ++i) {
+    float4 v = s[(i * 8) & 1023];
+    a.x += v.x; a.y += v.y; a.z += v.z; a.w += v.w;
+  }
+  if (a.x + a.y + a.z + a.w == 1.2345f) out[0] = a.x;
+}
+
+// ---- HBM streaming write (st.global.cs.v4) --------------------------------------
+__global__ void k_write(float4* __restrict__ dst, size_t n4) {
+  size_t stride = (size_t)gridDim.x * blockDim.x;
+  float4 v = make_float4(threadIdx.x, 1.f, 2.f, 3.f);
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) __stcs(dst + i, v);
+}
+
+int main() {
+  cudaDeviceProp p; CK(cudaGetDeviceProperties(&p, 0));
+  const int sms = p.multiProcessorCount;
+  float* dout; CK(cudaMalloc(&dout, 1 << 20));
+  unsigned long long* dclk; CK(cudaMalloc(&dclk, 2 * 8 * sms * sizeof(unsigned long long)));
+  cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+  const int threads = 256, blocks = sms * 8;   // 64 warps / SM
+  auto timeit = [&](auto launch) -> double {
+    launch(); cudaDeviceSynchronize();
+    cudaEventRecord(e0); for (int r = 0; r < 5; ++r) launch(); cudaEventRecord(e1);
+    cudaEventSynchronize(e1); float ms; cudaEventElapsedTime(&ms, e0, e1); return ms / 5 * 1e-3;
+  };
+  // clock
+  k_clock<<<sms, 128>>>(dclk, 1 << 22); CK(cudaDeviceSynchronize());
+  unsigned long long hclk[2]; CK(cudaMemcpy(hclk, dclk, sizeof(hclk), cudaMemcpyDeviceToHost));
+  double mhz = (double)hclk[0] / (double)hclk[1] * 1e3;
+  const double thr = (double)blocks * threads;
+  printf("{\"gpu\": \"%s\", \"sms\": %d, \"clock_mhz_busy\": %.1f", p.name, sms, mhz);
+  auto rep = [&](const char* name, double lane_ops, double sec) {
+    double per_s = lane_ops / sec;
+    printf(", \"%s\": {\"lane_ops_per_s\": %.4g, \"per_clk_per_sm\": %.2f}", name, per_s, per_s / (mhz * 1e6) / sms);
+  };
+  double it = (double)ITERS * 8 * thr;
+  rep("ffma", it, timeit([&] { k_ffma<<<blocks, threads>>>(dout, 0.999f, 0.001f); }));
+  rep("ffma2_lanes", 2 * it, timeit([&] { k_ffma2<<<blocks, threads>>>(dout, 0.999f, 0.001f); }));
+  rep("fadd", it, timeit([&] { k_fadd<<<blocks, threads>>>(dout, 0.001f); }));
+  rep("fadd2_lanes", 2 * it, timeit([&] { k_fadd2<<<blocks, threads>>>(dout, 0.001f); }));
+  rep("mufu_sqrt", it, timeit([&] { k_mufu<0><<<blocks, threads>>>(dout); }));
+  rep("mufu_rsqrt", it, timeit([&] { k_mufu<1><<<blocks, threads>>>(dout); }));
+  rep("mufu_ex2", it, timeit([&] { k_mufu<2><<<blocks, threads>>>(dout); }));
+  double at = (double)(ITERS / 4) * 8 * thr;
+  rep("atoms_lane_private", at, timeit([&] { k_atoms<0><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("atoms_random_256", at, timeit([&] { k_atoms<1><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("atoms_same_addr", at, timeit([&] { k_atoms<2><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("lds128_bcast_instr", (double)ITERS * thr, timeit([&] { k_lds128<<<blocks, threads>>>(dout); }));
+  size_t bytes = (size_t)8 << 30; float4* big; CK(cudaMalloc(&big, bytes));
+  double tw = timeit([&] { k_write<<<sms * 4, 512>>>(big, bytes / 16); });
+  printf(", \"hbm_write_stcs_GBps\": %.1f", bytes / tw * 1e-9);
+  double tm = timeit([&] { cudaMemsetAsync(big, 0, bytes); });
+  printf(", \"hbm_memset_GBps\": %.1f", bytes / tm * 1e-9);
+  // re-probe clock after the load
+  k_clock<<<sms, 128>>>(dclk, 1 << 22); CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(hclk, dclk, sizeof(hclk), cudaMemcpyDeviceToHost));
+  printf(", \"clock_mhz_busy_end\": %.1f}\n", (double)hclk[0] / (double)hclk[1] * 1e3);
+  CK(cudaGetLastError());
+  return 0;
+}
