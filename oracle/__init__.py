@@ -54,7 +54,8 @@ def _load():
         lib.oracle_sdh_lattice.argtypes = [_f32p, _i64, ctypes.c_int, _i64, ctypes.c_int, ctypes.c_int,
                                            _i64, _i64, _u64p]
         lib.oracle_pcf.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, _i64, _i64, _u64p, _u64p]
-        lib.oracle_pairmatrix.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, _i64, _i64, _f64p]
+        lib.oracle_pairmatrix.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_int, ctypes.c_double, _i64, _i64,
+                                          _f64p]
         lib.oracle_lattice_closed.argtypes = [_i64, _i64, ctypes.c_int, ctypes.c_int, _u64p, _i64, _u64p]
         lib.oracle_num_threads.restype = ctypes.c_int
         _lib = lib
@@ -123,12 +124,12 @@ def pcf(points, radius, rows=None):
     return int(c[0]), int(a[0])
 
 
-def pairmatrix(points, gamma, rows=None):
-    """Gaussian pair matrix rows [rb, re) x n in float64."""
+def pairmatrix(points, gamma, rows=None, ktype=0):
+    """Pair matrix rows [rb, re) x n in float64; ktype 0 Gaussian, 1 squared distance, 2 distance."""
     p, n, dim = _pts(points)
     rb, re = _rows(rows, n)
     out = np.zeros((re - rb, n), np.float64)
-    rc = _load().oracle_pairmatrix(_ptr(p, _f32p), n, dim, float(np.float32(gamma)), rb, re,
+    rc = _load().oracle_pairmatrix(_ptr(p, _f32p), n, dim, int(ktype), float(np.float32(gamma)), rb, re,
                                    _ptr(out, _f64p))
     if rc:
         raise ValueError(f"oracle_pairmatrix: status {rc}")

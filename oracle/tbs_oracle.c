@@ -178,17 +178,21 @@ int oracle_pcf(const float* P, int64_t n, int dim, double r, int64_t row_begin, 
 
 /*
  * Type-III pairwise-kernel matrix (L323-332, L709-712; reading Q10):
- * out[(i - row_begin) * n + j] = exp(-gamma * ||p_i - p_j||^2) for i in
- * [row_begin, row_end), all j in [0, n) (diagonal included).
+ * out[(i - row_begin) * n + j] = K(p_i, p_j) for i in [row_begin, row_end), all j in
+ * [0, n) (diagonal included), with K selected by ktype as in include/tbs.h:
+ *   0 Gaussian exp(-gamma * ||p_i - p_j||^2), 1 squared distance, 2 distance.
  */
-int oracle_pairmatrix(const float* P, int64_t n, int dim, double gamma, int64_t row_begin,
+int oracle_pairmatrix(const float* P, int64_t n, int dim, int ktype, double gamma, int64_t row_begin,
                       int64_t row_end, double* out) {
-  if (check_common(P, n, dim, row_begin, row_end) || !isfinite(gamma)) return ORACLE_EINVAL;
+  if (check_common(P, n, dim, row_begin, row_end) || !isfinite(gamma) || ktype < 0 || ktype > 2)
+    return ORACLE_EINVAL;
   if (row_end > row_begin && !out) return ORACLE_EINVAL;
 #pragma omp parallel for schedule(guided)
   for (int64_t i = row_begin; i < row_end; ++i)
-    for (int64_t j = 0; j < n; ++j)
-      out[(i - row_begin) * n + j] = exp(-gamma * dist2(P, dim, i, j));
+    for (int64_t j = 0; j < n; ++j) {
+      double s = dist2(P, dim, i, j);
+      out[(i - row_begin) * n + j] = ktype == 0 ? exp(-gamma * s) : ktype == 1 ? s : sqrt(s);
+    }
   return ORACLE_OK;
 }
 

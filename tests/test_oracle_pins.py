@@ -255,6 +255,10 @@ def test_pairmatrix_vs_cdist():
     assert np.all(np.diag(out) == 1.0)
     rows = oracle.pairmatrix(p, gamma, rows=(100, 140))
     assert np.array_equal(rows, out[100:140])
+    d2 = oracle.pairmatrix(p, 0.0, ktype=1)
+    np.testing.assert_allclose(d2, (d * d).numpy(), rtol=1e-13, atol=1e-300)
+    d1 = oracle.pairmatrix(p, 0.0, ktype=2)
+    np.testing.assert_allclose(d1, d.numpy(), rtol=1e-13, atol=1e-300)
 
 
 def test_pairmatrix_lattice_values():
