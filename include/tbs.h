@@ -41,7 +41,7 @@
  * nbuckets < 1 or > TBS_MAX_BUCKETS; bucket_width <= 0 or non-finite; radius < 0 or
  * NaN; NULL array with n >= 2 (or a NULL output); a row range outside [0, n];
  * TBS_EXACT_LATTICE with a bucket width that is not m * 2^-j (m, j integers,
- * 1 <= m < 2^20, 0 <= j <= 20). n < 2 (or an empty row range) is valid and yields
+ * 1 <= m, (nbuckets + 1) * m < 2^31, 0 <= j <= 19). n < 2 (or an empty row range) is valid and yields
  * zero output. Allocation failure returns TBS_ENOMEM; a CUDA error returns
  * TBS_ECUDA. tbs_last_error() gives a thread-local message for the last non-OK
  * status. Non-finite coordinates are a caller contract violation (not checked on

@@ -1,0 +1,223 @@
+"""B200-native 2-body statistics (Pitaksirianan, Nouri & Tu, ICPP 2016).
+
+Thin Python binding over the C ABI of ``libtbs.so`` (declared in include/tbs.h).
+Every step of the hot path runs in the library's sm_100a kernels; this module only
+marshals tensors (device pointers, the current CUDA stream) and, for multi-GPU,
+does the one collective of the method: ``all_reduce(SUM)`` of the per-rank
+histogram / count over NCCL. There is no CPU fallback: if the
+library or a CUDA device is missing, calls raise.
+
+    sdh(points, bucket_width, nbuckets)   Type-II spatial distance histogram (int64[nb])
+    pcf(points, radius)                   Type-I 2-point correlation count   (int64[1])
+    pairmatrix(points, gamma=1.0)         Type-III Gaussian pair matrix      (float32[rows, n])
+    rank_rows(n, world, rank)             pair-balanced anchor-row partition
+    sdh_host / pcf_host / pairmatrix_host the same through host (numpy) buffers
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libtbs.so")
+
+TBS_OK, TBS_EINVAL, TBS_ENOMEM, TBS_ECUDA, TBS_EUNSUPPORTED = range(5)
+TBS_EXACT_LATTICE = 0x1
+TBS_HIST_FORCE_LANE = 0x10
+TBS_HIST_FORCE_CTA = 0x20
+TBS_HIST_FORCE_GLOBAL = 0x40
+TBS_FORCE_CLAMP = 0x100
+KERNELS = {"gaussian": 0, "dist2": 1, "dist": 2}
+HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "global": TBS_HIST_FORCE_GLOBAL}
+
+# Symbols declared in include/tbs.h (checked by tests/test_abi.py).
+EXPORTS = ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
+           "tbs_rank_rows", "tbs_last_error", "tbs_release", "tbs_launch_count", "tbs_version")
+
+
+class TbsError(RuntimeError):
+    pass
+
+
+class _Args(ctypes.Structure):
+    _fields_ = [("points", ctypes.c_void_p), ("n", ctypes.c_int64), ("dim", ctypes.c_int),
+                ("row_begin", ctypes.c_int64), ("row_end", ctypes.c_int64), ("stream", ctypes.c_void_p),
+                ("flags", ctypes.c_uint32), ("ev_begin", ctypes.c_void_p), ("ev_end", ctypes.c_void_p)]
+
+
+class _Kernel(ctypes.Structure):
+    _fields_ = [("type", ctypes.c_int), ("gamma", ctypes.c_float)]
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libtbs.so (built in-tree by build.py / __graft_entry__.build()). Raises if missing."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise TbsError(f"{LIB_PATH} not built: run `python -m paper_conf_icpp_pitaksirianannt16_b200.build`")
+        L = ctypes.CDLL(LIB_PATH)
+        vp, i64, u64p = ctypes.c_void_p, ctypes.c_int64, ctypes.POINTER(ctypes.c_uint64)
+        L.tbs_sdh.argtypes = [vp, i64, ctypes.c_int, ctypes.c_float, ctypes.c_int, vp]
+        L.tbs_pcf.argtypes = [vp, i64, ctypes.c_float, vp]
+        L.tbs_pairmatrix.argtypes = [vp, i64, _Kernel, vp]
+        L.tbs_sdh_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_float, ctypes.c_int, vp]
+        L.tbs_pcf_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_float, vp]
+        L.tbs_pairmatrix_ex.argtypes = [ctypes.POINTER(_Args), _Kernel, vp]
+        L.tbs_rank_rows.argtypes = [i64, ctypes.c_int, ctypes.c_int, ctypes.POINTER(ctypes.c_int64),
+                                    ctypes.POINTER(ctypes.c_int64)]
+        L.tbs_last_error.restype = ctypes.c_char_p
+        L.tbs_launch_count.restype = ctypes.c_uint64
+        L.tbs_release.restype = None
+        for f in ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
+                  "tbs_rank_rows", "tbs_version"):
+            getattr(L, f).restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def _check(rc: int, what: str):
+    if rc != TBS_OK:
+        raise TbsError(f"{what}: status {rc}: {lib().tbs_last_error().decode()}")
+
+
+def last_error() -> str:
+    return lib().tbs_last_error().decode()
+
+
+def launch_count() -> int:
+    """Kernels libtbs.so has launched in this process."""
+    return int(lib().tbs_launch_count())
+
+
+def release() -> None:
+    lib().tbs_release()
+
+
+def version() -> int:
+    return int(lib().tbs_version())
+
+
+def rank_rows(n: int, world: int, rank: int) -> tuple[int, int]:
+    """Anchor rows of `rank` in the pair-count-balanced partition (host-only, no GPU)."""
+    b, e = ctypes.c_int64(), ctypes.c_int64()
+    _check(lib().tbs_rank_rows(int(n), int(world), int(rank), ctypes.byref(b), ctypes.byref(e)), "tbs_rank_rows")
+    return b.value, e.value
+
+
+# ---------------------------------------------------------------- device (torch) API
+def _torch():
+    import torch
+    return torch
+
+
+def _args(points, rows, flags, stream, events):
+    torch = _torch()
+    if not (isinstance(points, torch.Tensor) and points.is_cuda and points.dtype == torch.float32):
+        raise TypeError("points must be a CUDA float32 tensor [n, dim]")
+    if points.dim() == 1:
+        points = points.reshape(-1, 1)
+    if not points.is_contiguous():
+        raise ValueError("points must be contiguous (AoS [n][dim])")
+    n, dim = points.shape
+    rb, re = (0, n) if rows is None else (int(rows[0]), int(rows[1]))
+    st = stream if stream is not None else torch.cuda.current_stream(points.device)
+    a = _Args(points.data_ptr(), n, dim, rb, re, st.cuda_stream, flags, None, None)
+    if events is not None:
+        a.ev_begin, a.ev_end = events[0].cuda_event, events[1].cuda_event
+    return a, n
+
+
+def sdh(points, bucket_width: float, nbuckets: int, *, rows=None, lattice: bool = False, hist_mode=None,
+        force_clamp: bool = False, out=None, stream=None, events=None, group=None):
+    """Spatial distance histogram (Type-II). Returns int64[nbuckets] on points.device.
+
+    rows=(b, e): only anchors i in [b, e) (with all partners j > i). lattice=True:
+    exact integer bucketing (integer-valued points, bucket_width = m * 2^-j).
+    group: a torch.distributed process group: each rank computes its pair-balanced
+    strip (rank_rows) and the partial histograms are summed with one all_reduce.
+    """
+    torch = _torch()
+    flags = (TBS_EXACT_LATTICE if lattice else 0) | HIST_MODES[hist_mode] | (TBS_FORCE_CLAMP if force_clamp else 0)
+    if group is not None:
+        import torch.distributed as dist
+        rows = rank_rows(points.shape[0], dist.get_world_size(group), dist.get_rank(group))
+    a, _ = _args(points, rows, flags, stream, events)
+    h = out if out is not None else torch.empty(nbuckets, dtype=torch.int64, device=points.device)
+    _check(lib().tbs_sdh_ex(ctypes.byref(a), float(bucket_width), int(nbuckets), h.data_ptr()), "tbs_sdh_ex")
+    if group is not None:
+        import torch.distributed as dist
+        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+    return h
+
+
+def pcf(points, radius: float, *, rows=None, out=None, stream=None, events=None, group=None):
+    """2-point correlation count (Type-I): #{i<j : d < radius}, int64[1] on points.device."""
+    torch = _torch()
+    if group is not None:
+        import torch.distributed as dist
+        rows = rank_rows(points.shape[0], dist.get_world_size(group), dist.get_rank(group))
+    a, _ = _args(points, rows, 0, stream, events)
+    c = out if out is not None else torch.empty(1, dtype=torch.int64, device=points.device)
+    _check(lib().tbs_pcf_ex(ctypes.byref(a), float(radius), c.data_ptr()), "tbs_pcf_ex")
+    if group is not None:
+        import torch.distributed as dist
+        dist.all_reduce(c, op=dist.ReduceOp.SUM, group=group)
+    return c
+
+
+def pairmatrix(points, gamma: float = 1.0, *, kernel: str = "gaussian", rows=None, out=None, stream=None,
+               events=None, group=None):
+    """Type-III pair matrix rows [b, e) x n (float32). With a group, each rank gets its
+    block of rows (rank_rows over the full square is not needed: rows split evenly)."""
+    torch = _torch()
+    n = points.shape[0]
+    if group is not None:
+        import torch.distributed as dist
+        W, r = dist.get_world_size(group), dist.get_rank(group)
+        rows = (n * r // W, n * (r + 1) // W)
+    a, _ = _args(points, rows, 0, stream, events)
+    nr = a.row_end - a.row_begin
+    o = out if out is not None else torch.empty((nr, n), dtype=torch.float32, device=points.device)
+    _check(lib().tbs_pairmatrix_ex(ctypes.byref(a), _Kernel(KERNELS[kernel], float(gamma)), o.data_ptr()),
+           "tbs_pairmatrix_ex")
+    return o
+
+
+# ---------------------------------------------------------------- host (numpy) API
+def _host_points(points):
+    p = np.ascontiguousarray(points, dtype=np.float32)
+    if p.ndim == 1:
+        p = p.reshape(-1, 1)
+    return p
+
+
+def sdh_host(points, bucket_width: float, nbuckets: int, out=None):
+    """tbs_sdh with host buffers (H2D copy, kernels, D2H copy inside the call)."""
+    p = _host_points(points)
+    h = out if out is not None else np.empty(nbuckets, np.uint64)
+    _check(lib().tbs_sdh(p.ctypes.data, p.shape[0], p.shape[1], float(bucket_width), int(nbuckets), h.ctypes.data),
+           "tbs_sdh")
+    return h
+
+
+def pcf_host(points, radius: float) -> int:
+    p = _host_points(points)
+    assert p.shape[1] == 3
+    c = np.zeros(1, np.uint64)
+    _check(lib().tbs_pcf(p.ctypes.data, p.shape[0], float(radius), c.ctypes.data), "tbs_pcf")
+    return int(c[0])
+
+
+def pairmatrix_host(points, gamma: float = 1.0, kernel: str = "gaussian"):
+    p = _host_points(points)
+    assert p.shape[1] == 3
+    n = p.shape[0]
+    o = np.empty((n, n), np.float32)
+    _check(lib().tbs_pairmatrix(p.ctypes.data, n, _Kernel(KERNELS[kernel], float(gamma)), o.ctypes.data),
+           "tbs_pairmatrix")
+    return o

@@ -1,0 +1,461 @@
+// tbs_api.cu — the C-ABI host library (libtbs.so): argument validation, output-stage
+// selection, stream-ordered scratch, the work geometry, launches. Declared in
+// include/tbs.h (which cites the paper passages defining each operation).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "tbs.h"
+#include "tbs_kernels.cuh"
+
+using namespace tbs;
+
+namespace {
+
+thread_local std::string g_err;
+std::atomic<unsigned long long> g_launches{0};
+
+int fail(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+#define TBS_CUDA(call)                                                                        \
+  do {                                                                                        \
+    cudaError_t e_ = (call);                                                                  \
+    if (e_ != cudaSuccess) return fail(TBS_ECUDA, "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+  } while (0)
+
+struct Device {
+  int id = -1;
+  int sms = 0;
+  int smem_optin = 0;
+};
+
+int current_device(Device& d) {
+  int dev;
+  TBS_CUDA(cudaGetDevice(&dev));
+  static thread_local Device cache;
+  if (cache.id != dev) {
+    cudaDeviceProp p;
+    TBS_CUDA(cudaGetDeviceProperties(&p, dev));
+    cache.id = dev;
+    cache.sms = p.multiProcessorCount;
+    cache.smem_optin = (int)p.sharedMemPerBlockOptin;
+    // keep freed scratch cached in the stream-ordered pool (tbs_release() trims it)
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      unsigned long long thr = ~0ull;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
+  d = cache;
+  return TBS_OK;
+}
+
+// Persistent grid for a pair-kernel instantiation: SMs x resident CTAs (at most one CTA per item).
+template <class Op, int D>
+int launch_pair(const Device& dev, const float* soa, const Geom& g, const Op& op, cudaStream_t st, cudaEvent_t eb,
+                cudaEvent_t ee) {
+  auto kern = pair_kernel<Op, D>;
+  const long long smem = ((op.smem_bytes() + 127) & ~127ll) + 2ll * D * kTP * 4 + 16;
+  if (smem > dev.smem_optin) return fail(TBS_EUNSUPPORTED, "pair kernel needs %lld B smem > %d", smem, dev.smem_optin);
+  TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int occ = 0;
+  TBS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, (size_t)smem));
+  if (occ < 1) return fail(TBS_EUNSUPPORTED, "pair kernel cannot be resident (smem %lld)", smem);
+  long long grid = (long long)dev.sms * occ;
+  if (grid > g.items) grid = g.items;
+  if (eb) TBS_CUDA(cudaEventRecord(eb, st));
+  kern<<<(unsigned)grid, kThreads, (size_t)smem, st>>>(soa, g, op);
+  TBS_CUDA(cudaGetLastError());
+  g_launches.fetch_add(1);
+  if (ee) TBS_CUDA(cudaEventRecord(ee, st));
+  return TBS_OK;
+}
+
+Geom make_geom(int64_t n, int64_t rb, int64_t re) {
+  Geom g;
+  g.n = (int)n;
+  g.rb = (int)rb;
+  g.re = (int)re;
+  g.I0 = (int)(rb / kTA);
+  g.I1 = (int)((re + kTA - 1) / kTA);
+  g.Mc = (int)((n + kTP - 1) / kTP);
+  g.n_pad = (int)(((n + kTA - 1) / kTA) * kTA);
+  const long long I0 = g.I0, I1 = g.I1;
+  g.items = (I1 - I0) * (long long)g.Mc - (long long)kRatio * ((I1 * (I1 - 1) - I0 * (I0 - 1)) / 2);
+  return g;
+}
+
+int validate_common(const tbs_args* a) {
+  if (!a) return fail(TBS_EINVAL, "args is NULL");
+  if (a->n < 0 || a->n > TBS_MAX_N) return fail(TBS_EINVAL, "n = %lld outside [0, 2^30]", (long long)a->n);
+  if (a->dim < 1 || a->dim > 4) return fail(TBS_EINVAL, "dim = %d outside [1, 4]", a->dim);
+  if (a->row_begin < 0 || a->row_end < a->row_begin || a->row_end > a->n)
+    return fail(TBS_EINVAL, "row range [%lld, %lld) outside [0, %lld]", (long long)a->row_begin,
+                (long long)a->row_end, (long long)a->n);
+  if (a->n >= 2 && !a->points) return fail(TBS_EINVAL, "points is NULL");
+  return TBS_OK;
+}
+
+// SoA copy of the points in stream-ordered scratch; the loader also zeroes `zero` words.
+int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long long* zero, long long zero_words,
+                cudaStream_t st) {
+  TBS_CUDA(cudaMallocAsync((void**)soa, (size_t)D * n_pad * sizeof(float), st));
+  const int threads = 256;
+  long long blocks = std::min<long long>((n_pad + threads - 1) / threads, 148ll * 16);
+  blocks = std::max<long long>(blocks, 1);
+  soa_loader<<<(unsigned)blocks, threads, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, D, *soa, zero, zero_words);
+  TBS_CUDA(cudaGetLastError());
+  g_launches.fetch_add(1);
+  return TBS_OK;
+}
+
+// Decompose a dyadic width w = m * 2^-j (m odd or j = 0). Returns false if not dyadic.
+bool dyadic(float w, long long& m, int& j) {
+  double x = (double)w;
+  for (j = 0; j <= 19; ++j) {
+    double v = std::ldexp(x, j);
+    if (v == std::floor(v) && v >= 1.0 && v < 2147483648.0) {
+      m = (long long)v;
+      return true;
+    }
+  }
+  return false;
+}
+
+struct SdhPlan {
+  bool lattice, global;
+  int log2r;
+};
+
+template <int D, bool LAT>
+int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const Geom& g, float w, long long m, int j,
+                 int nb, unsigned long long* hist, unsigned long long* part, int G, cudaStream_t st, cudaEvent_t eb,
+                 cudaEvent_t ee) {
+  if (pl.global) {
+    SdhGlobalOp<LAT> op{};
+    op.nb = nb;
+    op.inv_w = (float)(1.0 / (double)w);
+    op.scale = (float)std::ldexp(1.0 / (double)m, j);
+    op.m = (int)m;
+    op.sh = 2 * j;
+    op.G = G;
+    op.part = part;
+    int rc = launch_pair<SdhGlobalOp<LAT>, D>(dev, soa, g, op, st, eb, ee);
+    if (rc) return rc;
+    reduce_partials<<<(nb + 255) / 256, 256, 0, st>>>(part, G, nb, hist);
+    TBS_CUDA(cudaGetLastError());
+    g_launches.fetch_add(1);
+    return TBS_OK;
+  }
+  auto fill = [&](auto& op, int R) {
+    op.nb = nb;
+    op.rows = nb;
+    op.inv_w = (float)(1.0 / (double)w);
+    op.scale = (float)std::ldexp(1.0 / (double)m, j);
+    op.m = (int)m;
+    op.sh = 2 * j;
+    op.hist = hist;
+    // per item, a replica receives at most (32/R) lanes x kWarps x kA x kTP increments
+    const long long per_item = (long long)(32 / R) * kWarps * kA * kTP;
+    op.flush_every = (int)std::max<long long>(1, (0xffffffffll / per_item) - 1);
+  };
+  switch (pl.log2r) {
+    case 5: { SdhSmemOp<5, LAT> op{}; fill(op, 32); return launch_pair<SdhSmemOp<5, LAT>, D>(dev, soa, g, op, st, eb, ee); }
+    case 2: { SdhSmemOp<2, LAT> op{}; fill(op, 4); return launch_pair<SdhSmemOp<2, LAT>, D>(dev, soa, g, op, st, eb, ee); }
+    default: { SdhSmemOp<0, LAT> op{}; fill(op, 1); return launch_pair<SdhSmemOp<0, LAT>, D>(dev, soa, g, op, st, eb, ee); }
+  }
+}
+
+int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
+  int rc = validate_common(a);
+  if (rc) return rc;
+  if (nb < 1 || nb > TBS_MAX_BUCKETS) return fail(TBS_EINVAL, "nbuckets = %d outside [1, 2^24]", nb);
+  if (!(w > 0.f) || !std::isfinite(w)) return fail(TBS_EINVAL, "bucket_width must be finite and > 0");
+  if (!hist) return fail(TBS_EINVAL, "hist is NULL");
+  const bool lattice = (a->flags & TBS_EXACT_LATTICE) != 0;
+  long long m = 1;
+  int j = 0;
+  if (lattice) {
+    if (!dyadic(w, m, j)) return fail(TBS_EINVAL, "TBS_EXACT_LATTICE needs bucket_width = m * 2^-j, j <= 19");
+    if ((long long)(nb + 1) * m >= (1ll << 31)) return fail(TBS_EINVAL, "TBS_EXACT_LATTICE needs (nb+1)*m < 2^31");
+  }
+  Device dev;
+  if ((rc = current_device(dev))) return rc;
+  cudaStream_t st = (cudaStream_t)a->stream;
+  auto* h = reinterpret_cast<unsigned long long*>(hist);
+  if (a->n < 2 || a->row_begin >= a->row_end) {
+    TBS_CUDA(cudaMemsetAsync(h, 0, (size_t)nb * 8, st));
+    return TBS_OK;
+  }
+  // Output-stage plan: lane-private copies (R = 32) while they fit a 96 KB budget (two CTAs
+  // per SM), then 4 replicas, then one copy per CTA; beyond that, global partial copies.
+  SdhPlan pl{lattice, false, 5};
+  const long long part_budget = std::min<long long>(96 * 1024, dev.smem_optin - 2ll * 4 * kTP * 4 - 256);
+  const long long one_copy_budget = dev.smem_optin - 2ll * 4 * kTP * 4 - 256;
+  if ((long long)nb * 32 * 4 <= part_budget) pl.log2r = 5;
+  else if ((long long)nb * 4 * 4 <= part_budget) pl.log2r = 2;
+  else if ((long long)nb * 4 <= one_copy_budget) pl.log2r = 0;
+  else pl.global = true;
+  if (a->flags & TBS_HIST_FORCE_LANE) {
+    if ((long long)nb * 32 * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_LANE: nb too large for smem");
+    pl = SdhPlan{lattice, false, 5};
+  }
+  if (a->flags & TBS_HIST_FORCE_CTA) {
+    if ((long long)nb * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_CTA: nb too large for smem");
+    pl = SdhPlan{lattice, false, 0};
+  }
+  if (a->flags & TBS_HIST_FORCE_GLOBAL) pl = SdhPlan{lattice, true, 0};
+
+  const int D = a->dim <= 3 ? 3 : 4;
+  const Geom g = make_geom(a->n, a->row_begin, a->row_end);
+  int G = 0;
+  unsigned long long* part = nullptr;
+  long long zero_words = 0;
+  if (pl.global) {
+    G = std::min(dev.sms, 64);
+    TBS_CUDA(cudaMallocAsync((void**)&part, (size_t)G * nb * 8, st));
+    zero_words = (long long)G * nb;
+  }
+  float* soa = nullptr;
+  // Smem modes accumulate into hist: the loader zeroes it. Global mode zeroes the partials
+  // (the reduce kernel overwrites hist).
+  rc = load_points(a, D, g.n_pad, &soa, pl.global ? part : h, pl.global ? zero_words : nb, st);
+  if (!rc) {
+    cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
+    if (D == 3) rc = lattice ? sdh_dispatch<3, true>(dev, pl, soa, g, w, m, j, nb, h, part, G, st, eb, ee)
+                             : sdh_dispatch<3, false>(dev, pl, soa, g, w, m, j, nb, h, part, G, st, eb, ee);
+    else rc = lattice ? sdh_dispatch<4, true>(dev, pl, soa, g, w, m, j, nb, h, part, G, st, eb, ee)
+                      : sdh_dispatch<4, false>(dev, pl, soa, g, w, m, j, nb, h, part, G, st, eb, ee);
+  }
+  if (soa) cudaFreeAsync(soa, st);
+  if (part) cudaFreeAsync(part, st);
+  return rc;
+}
+
+int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
+  int rc = validate_common(a);
+  if (rc) return rc;
+  if (!(r >= 0.f) || std::isinf(r)) return fail(TBS_EINVAL, "radius must be finite and >= 0");
+  if (!count) return fail(TBS_EINVAL, "count is NULL");
+  Device dev;
+  if ((rc = current_device(dev))) return rc;
+  cudaStream_t st = (cudaStream_t)a->stream;
+  auto* c = reinterpret_cast<unsigned long long*>(count);
+  if (a->n < 2 || a->row_begin >= a->row_end) {
+    TBS_CUDA(cudaMemsetAsync(c, 0, 8, st));
+    return TBS_OK;
+  }
+  const int D = a->dim <= 3 ? 3 : 4;
+  const Geom g = make_geom(a->n, a->row_begin, a->row_end);
+  float* soa = nullptr;
+  rc = load_points(a, D, g.n_pad, &soa, c, 1, st);
+  if (!rc) {
+    PcfOp op{};
+    op.r2 = (float)((double)r * (double)r);
+    op.count = c;
+    cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
+    rc = D == 3 ? launch_pair<PcfOp, 3>(dev, soa, g, op, st, eb, ee) : launch_pair<PcfOp, 4>(dev, soa, g, op, st, eb, ee);
+  }
+  if (soa) cudaFreeAsync(soa, st);
+  return rc;
+}
+
+template <int KT, int D>
+int matrix_launch(const tbs_args* a, const float* soa, int n_pad, float cexp, float* out, cudaStream_t st) {
+  const int n = (int)a->n;
+  dim3 grid((unsigned)((n + kMatCols - 1) / kMatCols), (unsigned)((a->row_end - a->row_begin + kMatRows - 1) / kMatRows));
+  if (grid.y > 2147483647u) return fail(TBS_EUNSUPPORTED, "too many rows");
+  cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
+  if (eb) TBS_CUDA(cudaEventRecord(eb, st));
+  if (n % 4 == 0)
+    pairmatrix_kernel<KT, D, true><<<grid, kMatThreads, 0, st>>>(soa, n, n_pad, (int)a->row_begin, (int)a->row_end, cexp, out);
+  else
+    pairmatrix_kernel<KT, D, false><<<grid, kMatThreads, 0, st>>>(soa, n, n_pad, (int)a->row_begin, (int)a->row_end, cexp, out);
+  TBS_CUDA(cudaGetLastError());
+  g_launches.fetch_add(1);
+  if (ee) TBS_CUDA(cudaEventRecord(ee, st));
+  return TBS_OK;
+}
+
+int pairmatrix_impl(const tbs_args* a, tbs_kernel k, float* out) {
+  int rc = validate_common(a);
+  if (rc) return rc;
+  if (k.type < 0 || k.type > 2) return fail(TBS_EINVAL, "kernel type %d unknown", k.type);
+  if (k.type == TBS_K_GAUSSIAN && !std::isfinite(k.gamma)) return fail(TBS_EINVAL, "gamma must be finite");
+  if (a->row_end > a->row_begin && !out) return fail(TBS_EINVAL, "out is NULL");
+  if (a->row_end == a->row_begin || a->n == 0) return TBS_OK;
+  cudaStream_t st = (cudaStream_t)a->stream;
+  const int D = a->dim <= 3 ? 3 : 4;
+  const int n_pad = (int)(((a->n + kTA - 1) / kTA) * kTA);
+  float* soa = nullptr;
+  rc = load_points(a, D, n_pad, &soa, nullptr, 0, st);
+  if (!rc) {
+    const float cexp = (float)(-(double)k.gamma * 1.4426950408889634);  // -gamma * log2(e)
+    if (D == 3) rc = k.type == 0 ? matrix_launch<0, 3>(a, soa, n_pad, cexp, out, st)
+                     : k.type == 1 ? matrix_launch<1, 3>(a, soa, n_pad, cexp, out, st)
+                                   : matrix_launch<2, 3>(a, soa, n_pad, cexp, out, st);
+    else rc = k.type == 0 ? matrix_launch<0, 4>(a, soa, n_pad, cexp, out, st)
+              : k.type == 1 ? matrix_launch<1, 4>(a, soa, n_pad, cexp, out, st)
+                            : matrix_launch<2, 4>(a, soa, n_pad, cexp, out, st);
+  }
+  if (soa) cudaFreeAsync(soa, st);
+  return rc;
+}
+
+// ---- host-or-device simple entry points ------------------------------------------
+int is_device_ptr(const void* p, bool& dev) {
+  dev = false;
+  if (!p) return TBS_OK;
+  cudaPointerAttributes at;
+  cudaError_t e = cudaPointerGetAttributes(&at, p);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return TBS_OK;  // unregistered host memory
+  }
+  dev = at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+  return TBS_OK;
+}
+
+// Run `fn(args_with_device_ptrs, dev_out)` for host or device buffers, synchronously.
+template <class Fn>
+int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_bytes, Fn fn) {
+  if (n < 0 || n > TBS_MAX_N) return fail(TBS_EINVAL, "n out of range");
+  if (dim < 1 || dim > 4) return fail(TBS_EINVAL, "dim out of range");
+  if (!outp) return fail(TBS_EINVAL, "output is NULL");
+  if (n >= 2 && !points) return fail(TBS_EINVAL, "points is NULL");
+  bool pdev = false, odev = false;
+  int rc = is_device_ptr(points, pdev);
+  if (!rc) rc = is_device_ptr(outp, odev);
+  if (rc) return rc;
+  if (points && pdev != odev) return fail(TBS_EINVAL, "points and output must both be host or both device pointers");
+  cudaStream_t st = cudaStreamPerThread;
+  tbs_args a{};
+  a.n = n;
+  a.dim = dim;
+  a.row_begin = 0;
+  a.row_end = n;
+  a.stream = st;
+  if (odev) {
+    a.points = points;
+    rc = fn(&a, outp);
+    if (!rc) TBS_CUDA(cudaStreamSynchronize(st));
+    return rc;
+  }
+  float* dp = nullptr;
+  void* dout = nullptr;
+  const size_t pbytes = (size_t)n * dim * sizeof(float);
+  if (pbytes) TBS_CUDA(cudaMallocAsync((void**)&dp, pbytes, st));
+  cudaError_t e = cudaMallocAsync(&dout, out_bytes, st);
+  if (e != cudaSuccess) {
+    if (dp) cudaFreeAsync(dp, st);
+    return fail(TBS_ENOMEM, "cudaMallocAsync(%zu): %s", out_bytes, cudaGetErrorString(e));
+  }
+  if (pbytes) e = cudaMemcpyAsync(dp, points, pbytes, cudaMemcpyHostToDevice, st);
+  a.points = dp;
+  rc = e != cudaSuccess ? fail(TBS_ECUDA, "H2D copy: %s", cudaGetErrorString(e)) : fn(&a, dout);
+  if (!rc) {
+    e = cudaMemcpyAsync(outp, dout, out_bytes, cudaMemcpyDeviceToHost, st);
+    if (e != cudaSuccess) rc = fail(TBS_ECUDA, "D2H copy: %s", cudaGetErrorString(e));
+  }
+  if (dp) cudaFreeAsync(dp, st);
+  cudaFreeAsync(dout, st);
+  e = cudaStreamSynchronize(st);
+  if (!rc && e != cudaSuccess) rc = fail(TBS_ECUDA, "sync: %s", cudaGetErrorString(e));
+  return rc;
+}
+
+}  // namespace
+
+extern "C" {
+
+int tbs_sdh_ex(const tbs_args* args, float bucket_width, int nbuckets, uint64_t* hist) {
+  g_err.clear();
+  return sdh_impl(args, bucket_width, nbuckets, hist);
+}
+
+int tbs_pcf_ex(const tbs_args* args, float radius, uint64_t* count) {
+  g_err.clear();
+  return pcf_impl(args, radius, count);
+}
+
+int tbs_pairmatrix_ex(const tbs_args* args, tbs_kernel kernel, float* out) {
+  g_err.clear();
+  return pairmatrix_impl(args, kernel, out);
+}
+
+int tbs_sdh(const float* points, int64_t n, int dim, float bucket_width, int nbuckets, uint64_t* hist) {
+  g_err.clear();
+  if (nbuckets < 1 || nbuckets > TBS_MAX_BUCKETS) return fail(TBS_EINVAL, "nbuckets out of range");
+  return run_simple(points, n, dim, hist, (size_t)nbuckets * 8, [&](tbs_args* a, void* out) {
+    return sdh_impl(a, bucket_width, nbuckets, (uint64_t*)out);
+  });
+}
+
+int tbs_pcf(const float* points, int64_t n, float radius, uint64_t* count) {
+  g_err.clear();
+  return run_simple(points, n, 3, count, 8, [&](tbs_args* a, void* out) { return pcf_impl(a, radius, (uint64_t*)out); });
+}
+
+int tbs_pairmatrix(const float* points, int64_t n, tbs_kernel kernel, float* out) {
+  g_err.clear();
+  if (n < 0 || n > TBS_MAX_N) return fail(TBS_EINVAL, "n out of range");
+  return run_simple(points, n, 3, out, (size_t)n * (size_t)n * sizeof(float) + (n == 0 ? 4 : 0),
+                    [&](tbs_args* a, void* o) { return pairmatrix_impl(a, kernel, (float*)o); });
+}
+
+int tbs_rank_rows(int64_t n, int world, int rank, int64_t* row_begin, int64_t* row_end) {
+  g_err.clear();
+  if (n < 0 || world < 1 || rank < 0 || rank >= world || !row_begin || !row_end)
+    return fail(TBS_EINVAL, "tbs_rank_rows: bad arguments");
+  // S(R) = sum_{i<R} (n-1-i) = R(2n-R-1)/2 pairs have anchors below row R. Boundary r
+  // solves S(R) = r * P / world, P = n(n-1)/2; take the integer R whose S is nearest.
+  auto boundary = [&](int r) -> int64_t {
+    if (r <= 0) return 0;
+    if (r >= world) return n;
+    const __int128 P = (__int128)n * (n - 1) / 2;
+    const __int128 target = P * r / world;
+    const double b = 2.0 * (double)n - 1.0;
+    double R = 0.5 * (b - std::sqrt(std::max(0.0, b * b - 8.0 * (double)target)));
+    int64_t Ri = std::min<int64_t>(std::max<int64_t>((int64_t)R, 0), n);
+    auto S = [&](int64_t x) { return (__int128)x * (2 * n - x - 1) / 2; };
+    while (Ri > 0 && S(Ri) > target) --Ri;
+    while (Ri < n && S(Ri + 1) <= target) ++Ri;
+    if (Ri < n && (S(Ri + 1) - target) < (target - S(Ri))) ++Ri;
+    return Ri;
+  };
+  *row_begin = boundary(rank);
+  *row_end = boundary(rank + 1);
+  return TBS_OK;
+}
+
+const char* tbs_last_error(void) { return g_err.c_str(); }
+
+void tbs_release(void) {
+  int dev;
+  if (cudaGetDevice(&dev) != cudaSuccess) return;
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    cudaDeviceSynchronize();
+    cudaMemPoolTrimTo(pool, 0);
+  }
+}
+
+uint64_t tbs_launch_count(void) { return g_launches.load(); }
+
+int tbs_version(void) { return 100; }
+
+}  // extern "C"

@@ -1,0 +1,437 @@
+// tbs_kernels.cuh — sm_100a kernels of the 2-body-statistics hot path.
+//
+// Paper: Pitaksirianan, Nouri & Tu, ICPP 2016 (/root/reference/PAPER.md, cited L<a>-<b>).
+// The design keeps the paper's ideas that still hold on B200 and drops the rest
+// (DESIGN.md §Kernels):
+//   * SoA input (L338-341)                       -> loader writes [D][n_pad] fp32 SoA
+//   * block tiling, Alg. 2 (L366-458)            -> triangular (anchor tile, partner chunk)
+//                                                   work items over persistent CTAs
+//   * anchor datum in registers, Alg. 3 (L465-511)-> kA = 8 anchors per thread, packed in
+//                                                   f32x2 register pairs (FADD2/FFMA2)
+//   * partner block in cache (L499)              -> TMA bulk copy (cp.async.bulk) into
+//                                                   shared memory, double-buffered on mbarriers,
+//                                                   read as LDS.128 broadcasts
+//   * privatised output, Fig. 3 (L722-782)       -> 32 lane-private u32 copies per CTA
+//                                                   (conflict-free ATOMS), u64 flush
+//   * Type-I register output (L704-709)          -> per-thread sign-bit counter
+//   * Type-III global output (L709-712)          -> streaming float4 stores
+//   * intra-block i<j (Alg. 2 l.9-12, Fig. 6)    -> predicated pairs on diagonal items
+#pragma once
+#include <cstdint>
+#include "tbs_ptx.cuh"
+
+namespace tbs {
+
+constexpr int kThreads = 256;              // 8 warps per CTA
+constexpr int kWarps = kThreads / 32;
+constexpr int kA = 8;                      // anchors per thread (4 f32x2 pairs)
+constexpr int kTA = kThreads * kA;         // anchor tile: 2048 points
+constexpr int kTP = 1024;                  // partner chunk: 1024 points
+constexpr int kRatio = kTA / kTP;          // partner chunks per anchor tile
+constexpr uint32_t kMagic = 0x4B000000u;   // bits of 2^23: x + 2^23 (round-down) = 2^23 + floor(x)
+constexpr float kMagicF = 8388608.0f;
+constexpr int kNoAnchor = 0x7fffffff;      // masked anchor index (no partner is greater)
+
+// Work decomposition (host-computed). Anchor tiles I in [I0, I1) of kTA points; for each,
+// partner chunks J in [I*kRatio, Mc) of kTP points. Item count: sum_I (Mc - I*kRatio).
+struct Geom {
+  int n;            // number of points
+  int rb, re;       // anchor rows [rb, re)
+  int I0, I1;       // anchor tiles
+  int Mc;           // ceil(n / kTP)
+  int n_pad;        // SoA row stride (multiple of kTA)
+  long long items;  // total work items
+};
+
+__device__ __forceinline__ long long items_before(const Geom& g, long long I) {
+  return (I - g.I0) * (long long)g.Mc - (long long)kRatio * ((I * (I - 1) - (long long)g.I0 * (g.I0 - 1)) / 2);
+}
+__device__ __forceinline__ void item_to_tile(const Geom& g, long long it, int& I, int& J) {
+  int lo = g.I0, hi = g.I1 - 1;
+  while (lo < hi) {
+    int mid = (lo + hi + 1) >> 1;
+    if (items_before(g, mid) <= it) lo = mid; else hi = mid - 1;
+  }
+  I = lo;
+  J = lo * kRatio + (int)(it - items_before(g, lo));
+}
+
+// ------------------------------------------------------------------------------------
+// a1: SoA loader. AoS [n][dim] -> SoA [D][n_pad] (pad coordinates and pad points = 0).
+// Also zeroes `zero_words` u64 words at `zero` (the caller's output / partial copies),
+// saving a separate memset launch.
+// ------------------------------------------------------------------------------------
+__global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_pad, int D,
+                           float* __restrict__ soa, unsigned long long* __restrict__ zero, long long zero_words) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n_pad; i += stride) {
+    for (int c = 0; c < D; ++c)
+      soa[(long long)c * n_pad + i] = (i < n && c < dim) ? __ldg(pts + i * dim + c) : 0.0f;
+  }
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < zero_words; i += stride) zero[i] = 0ull;
+}
+
+// ------------------------------------------------------------------------------------
+// Output-stage policies. Each provides:
+//   smem_bytes()                    dynamic shared memory it needs (host and device)
+//   init(smem), finish(smem)        zero / flush its private copies
+//   after_item(smem, since)         flush early if a u32 counter could overflow
+//   bias()                          value the squared-distance chain starts from
+//   pair2<MASKED>(s2, pv, a0, a1)   consume two pairs (anchors a0, a1 vs partner pv);
+//                                   under MASKED a pair counts only if pv > a
+// ------------------------------------------------------------------------------------
+
+// Type-II, float mode: bucket = min(floor(sqrt(s) / w), nb - 1) with R replicas per bin
+// in shared memory, layout word[k * R + (lane & (R-1))]. R = 32: every lane owns a copy
+// and the 32 lanes of an ATOMS hit 32 distinct banks (no conflicts, no same-address).
+// LATTICE: exact integer bucketing max{k : (k m)^2 <= 4^j s} for integer-valued input.
+template <int LOG2R, bool LATTICE>
+struct SdhSmemOp {
+  static constexpr int R = 1 << LOG2R;
+  int nb;             // buckets
+  int rows;           // rows allocated (= nb)
+  float inv_w;        // fp32(1 / w)                       (float mode)
+  float scale;        // fp32(2^j / m)                     (lattice mode)
+  int m, sh;          // w = m * 2^-j, sh = 2 j            (lattice mode)
+  unsigned long long* hist;  // global u64 output [nb]
+  uint32_t base;      // shared address of word 0 for this lane, minus the magic offset
+  uint32_t bmax;      // magic bits of bucket nb-1 (clamp)
+  int flush_every;    // items between overflow flushes
+
+  __host__ __device__ long long smem_bytes() const { return (long long)rows * R * 4; }
+
+  __device__ __forceinline__ void init(unsigned char* smem) {
+    uint32_t* h = reinterpret_cast<uint32_t*>(smem);
+    for (int i = threadIdx.x; i < rows * R; i += kThreads) h[i] = 0u;
+    const int lane = threadIdx.x & 31;
+    base = smem_addr(smem) + (uint32_t)((lane & (R - 1)) * 4) - (kMagic << (LOG2R + 2));
+    bmax = kMagic + (uint32_t)(nb - 1);
+  }
+  __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
+
+  __device__ __forceinline__ uint32_t bucket_bits(float s) const {
+    if (!LATTICE) {
+      return 0u;  // unused (packed path below)
+    } else {
+      // s is an exact integer < 2^24. fp32 estimate, then exact integer fix-up by one step.
+      uint32_t si = __float2uint_rz(s);
+      float q = sqrt_approx(s);
+      int k = min((int)(__float_as_uint(__fmaf_rd(q, scale, kMagicF)) - kMagic), nb);
+      unsigned long long S = (unsigned long long)si << sh;
+      unsigned long long e1 = (unsigned long long)(k + 1) * (unsigned long long)m;
+      k += (e1 * e1 <= S) ? 1 : 0;
+      unsigned long long e0 = (unsigned long long)k * (unsigned long long)m;
+      k -= (e0 * e0 > S) ? 1 : 0;
+      return kMagic + (uint32_t)k;
+    }
+  }
+
+  template <bool MASKED>
+  __device__ __forceinline__ void pair2(float2 s, int pv, int a0, int a1) {
+    uint32_t b0, b1;
+    if (!LATTICE) {
+      // floor(sqrt(s) * inv_w) via one FFMA2.RM onto 2^23: the scale and the floor in one op
+      float2 q = make_float2(sqrt_approx(s.x), sqrt_approx(s.y));
+      float2 k = __ffma2_rd(q, make_float2(inv_w, inv_w), make_float2(kMagicF, kMagicF));
+      b0 = __float_as_uint(k.x);
+      b1 = __float_as_uint(k.y);
+    } else {
+      b0 = bucket_bits(s.x);
+      b1 = bucket_bits(s.y);
+    }
+    b0 = min(b0, bmax);
+    b1 = min(b1, bmax);
+    const uint32_t ad0 = (b0 << (LOG2R + 2)) + base, ad1 = (b1 << (LOG2R + 2)) + base;
+    if (MASKED) {
+      red_smem_inc_gt(ad0, pv, a0);
+      red_smem_inc_gt(ad1, pv, a1);
+    } else {
+      red_smem_inc(ad0);
+      red_smem_inc(ad1);
+    }
+  }
+
+  // Sum the R replicas of each bin (segmented shuffle) and add to the global u64 output.
+  __device__ void flush(unsigned char* smem) {
+    uint32_t* h = reinterpret_cast<uint32_t*>(smem);
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int total = rows * R;
+    for (int e0 = warp * 32; e0 < total; e0 += kWarps * 32) {
+      const int e = e0 + lane;
+      unsigned long long v = 0;
+      if (e < total) { v = h[e]; h[e] = 0u; }
+#pragma unroll
+      for (int off = 1; off < R; off <<= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+      if ((lane & (R - 1)) == 0 && v != 0ull && e < total) {
+        int k = e >> LOG2R;
+        atomicAdd(hist + (k < nb ? k : nb - 1), v);
+      }
+    }
+  }
+  __device__ __forceinline__ void after_item(unsigned char* smem, int& since) {
+    if (++since >= flush_every) {
+      flush(smem);
+      __syncthreads();
+      since = 0;
+    }
+  }
+  __device__ __forceinline__ void finish(unsigned char* smem) { flush(smem); }
+};
+
+// Type-II, partially privatised GLOBAL histogram (large nb, or forced): G u64 copies in
+// global memory (L2-resident), CTA b adds into copy b % G; a reduce kernel sums them.
+template <bool LATTICE>
+struct SdhGlobalOp {
+  int nb;
+  float inv_w, scale;
+  int m, sh;
+  int G;
+  unsigned long long* part;  // [G][nb]
+  unsigned long long* mine;
+  int flush_every;           // unused
+
+  __host__ __device__ long long smem_bytes() const { return 0; }
+  __device__ __forceinline__ void init(unsigned char*) { mine = part + (size_t)(blockIdx.x % G) * nb; }
+  __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
+  __device__ __forceinline__ int bucket(float s) const {
+    int k;
+    if (!LATTICE) {
+      k = (int)(__float_as_uint(__fmaf_rd(sqrt_approx(s), inv_w, kMagicF)) - kMagic);
+    } else {
+      uint32_t si = __float2uint_rz(s);
+      k = min((int)(__float_as_uint(__fmaf_rd(sqrt_approx(s), scale, kMagicF)) - kMagic), nb);
+      unsigned long long S = (unsigned long long)si << sh;
+      unsigned long long e1 = (unsigned long long)(k + 1) * (unsigned long long)m;
+      k += (e1 * e1 <= S) ? 1 : 0;
+      unsigned long long e0 = (unsigned long long)k * (unsigned long long)m;
+      k -= (e0 * e0 > S) ? 1 : 0;
+    }
+    return min(k, nb - 1);
+  }
+  template <bool MASKED>
+  __device__ __forceinline__ void pair2(float2 s, int pv, int a0, int a1) {
+    unsigned long long* p0 = mine + bucket(s.x);
+    unsigned long long* p1 = mine + bucket(s.y);
+    if (MASKED) {
+      red_gmem_inc64_gt(p0, pv, a0);
+      red_gmem_inc64_gt(p1, pv, a1);
+    } else {
+      red_gmem_inc64(p0);
+      red_gmem_inc64(p1);
+    }
+  }
+  __device__ __forceinline__ void after_item(unsigned char*, int&) {}
+  __device__ __forceinline__ void finish(unsigned char*) {}
+};
+
+// Type-I 2PCF count: t = s - r^2 is formed inside the FMA chain (bias = -r^2), and the
+// count adds the sign bit of t: [s < r^2] with no compare instruction.
+struct PcfOp {
+  float r2;
+  unsigned long long* count;
+  uint32_t c;                // per-item counter (<= kA * kTP)
+  unsigned long long total;  // per-thread running total
+
+  __host__ __device__ long long smem_bytes() const { return 0; }
+  __device__ __forceinline__ void init(unsigned char*) { c = 0u; total = 0ull; }
+  __device__ __forceinline__ float2 bias() const { return make_float2(-r2, -r2); }
+  template <bool MASKED>
+  __device__ __forceinline__ void pair2(float2 t, int pv, int a0, int a1) {
+    uint32_t s0 = __float_as_uint(t.x) >> 31, s1 = __float_as_uint(t.y) >> 31;
+    if (MASKED) {
+      s0 = (pv > a0) ? s0 : 0u;
+      s1 = (pv > a1) ? s1 : 0u;
+    }
+    c += s0 + s1;
+  }
+  __device__ __forceinline__ void after_item(unsigned char*, int&) {
+    total += c;
+    c = 0u;
+  }
+  __device__ void finish(unsigned char* smem) {
+    total += c;
+    unsigned long long v = total;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+    unsigned long long* red = reinterpret_cast<unsigned long long*>(smem);  // >= kWarps * 8 bytes (partner buffers)
+    __syncthreads();
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long s = 0;
+      for (int w = 0; w < kWarps; ++w) s += red[w];
+      if (s) atomicAdd(count, s);
+    }
+  }
+};
+
+// ------------------------------------------------------------------------------------
+// a2-a10: the pair engine. Persistent CTAs walk a contiguous range of the linearised
+// triangular item list. Per item: anchors (kA per thread) in registers, partner chunk
+// staged by TMA into a double-buffered smem slot, every (anchor, partner) pair evaluated
+// as packed f32x2 arithmetic, the Op consumes the squared distances.
+// ------------------------------------------------------------------------------------
+template <class Op, int D>
+__device__ __forceinline__ void issue_chunk(const float* __restrict__ soa, const Geom& g, int J, float* dst,
+                                            uint32_t bar) {
+  mbar_arrive_expect_tx(bar, D * kTP * 4);
+#pragma unroll
+  for (int c = 0; c < D; ++c)
+    bulk_g2s(smem_addr(dst + c * kTP), soa + (long long)c * g.n_pad + (long long)J * kTP, kTP * 4, bar);
+}
+
+template <class Op, int D, bool MASKED>
+__device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, const float2 (&na)[D][kA / 2],
+                                          const int (&aidx)[kA], int p0, int cnt, int n) {
+  for (int p = 0; p < cnt; p += 4) {
+    float c4[D][4];
+#pragma unroll
+    for (int c = 0; c < D; ++c) {
+      const float4 v = *reinterpret_cast<const float4*>(B + c * kTP + p);
+      c4[c][0] = v.x; c4[c][1] = v.y; c4[c][2] = v.z; c4[c][3] = v.w;
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      int pv = 0;
+      if (MASKED) pv = (p0 + p + q < n) ? p0 + p + q : -1;
+#pragma unroll
+      for (int m = 0; m < kA / 2; ++m) {
+        float2 d = __fadd2_rn(na[0][m], make_float2(c4[0][q], c4[0][q]));
+        float2 s = __ffma2_rn(d, d, op.bias());
+#pragma unroll
+        for (int c = 1; c < D; ++c) {
+          d = __fadd2_rn(na[c][m], make_float2(c4[c][q], c4[c][q]));
+          s = __ffma2_rn(d, d, s);
+        }
+        op.template pair2<MASKED>(s, pv, aidx[2 * m], aidx[2 * m + 1]);
+      }
+    }
+  }
+}
+
+template <class Op, int D>
+__global__ void __launch_bounds__(kThreads, 2) pair_kernel(const float* __restrict__ soa, Geom g, Op op) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  const long long hbytes = (op.smem_bytes() + 127) & ~127ll;
+  float* bufs = reinterpret_cast<float*>(smem + hbytes);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + hbytes + 2 * D * kTP * 4);
+  const uint32_t bar0 = smem_addr(bars), bar1 = smem_addr(bars + 1);
+  const int tid = threadIdx.x;
+
+  op.init(smem);
+  if (tid == 0) {
+    mbar_init(bar0, 1);
+    mbar_init(bar1, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+
+  const long long beg = (g.items * (long long)blockIdx.x) / gridDim.x;
+  const long long end = (g.items * (long long)(blockIdx.x + 1)) / gridDim.x;
+  if (beg < end) {
+    int I, J;
+    item_to_tile(g, beg, I, J);
+    if (tid == 0) issue_chunk<Op, D>(soa, g, J, bufs, bar0);
+    int curI = -1;
+    uint32_t phase = 0u;  // bit s = parity of buffer s
+    int since = 0;
+    float2 na[D][kA / 2];  // negated anchor coordinates, packed (a_{2m}, a_{2m+1})
+    int aidx[kA];          // anchor index, or kNoAnchor if outside [rb, re)
+    for (long long it = beg; it < end; ++it) {
+      const int s = (int)((it - beg) & 1);
+      int nI = I, nJ = J + 1;
+      if (nJ == g.Mc) { nI = I + 1; nJ = nI * kRatio; }
+      if (tid == 0 && it + 1 < end) issue_chunk<Op, D>(soa, g, nJ, bufs + (s ^ 1) * D * kTP, s ? bar0 : bar1);
+      if (I != curI) {
+        curI = I;
+#pragma unroll
+        for (int k = 0; k < kA; ++k) {
+          const int a = I * kTA + k * kThreads + tid;
+          aidx[k] = (a >= g.rb && a < g.re) ? a : kNoAnchor;
+#pragma unroll
+          for (int c = 0; c < D; ++c) {
+            const float v = -__ldg(soa + (long long)c * g.n_pad + a);
+            if (k & 1) na[c][k >> 1].y = v; else na[c][k >> 1].x = v;
+          }
+        }
+      }
+      mbar_wait(s ? bar1 : bar0, (phase >> s) & 1u);
+      phase ^= 1u << s;
+      const float* B = bufs + s * D * kTP;
+      const int p0 = J * kTP;
+      const int cnt = min(kTP, g.n - p0);
+      const bool fast = (I * kTA >= g.rb) && ((I + 1) * kTA <= g.re) && (p0 >= (I + 1) * kTA) && (cnt == kTP);
+      if (fast) run_chunk<Op, D, false>(op, B, na, aidx, p0, cnt, g.n);
+      else run_chunk<Op, D, true>(op, B, na, aidx, p0, cnt, g.n);
+      __syncthreads();
+      op.after_item(smem, since);
+      I = nI;
+      J = nJ;
+    }
+  }
+  __syncthreads();
+  op.finish(smem);
+}
+
+// Sum G partial global copies into the output (one thread per bin, the paper's
+// reduction kernel K13, L778-782).
+__global__ void reduce_partials(const unsigned long long* __restrict__ part, int G, int nb,
+                                unsigned long long* __restrict__ hist) {
+  for (int k = blockIdx.x * blockDim.x + threadIdx.x; k < nb; k += gridDim.x * blockDim.x) {
+    unsigned long long s = 0;
+    for (int gi = 0; gi < G; ++gi) s += part[(size_t)gi * nb + k];
+    hist[k] = s;
+  }
+}
+
+// ------------------------------------------------------------------------------------
+// a11: Type-III pair matrix. Each thread owns 4 consecutive columns (registers) and
+// walks kMatRows rows whose coordinates are warp-uniform loads; each row writes one
+// float4 per thread with a streaming store: a warp writes 512 contiguous bytes.
+// ------------------------------------------------------------------------------------
+constexpr int kMatThreads = 256;
+constexpr int kMatCols = kMatThreads * 4;  // 1024 columns per CTA
+constexpr int kMatRows = 16;               // rows per CTA
+
+template <int KTYPE, int D, bool VEC>
+__global__ void __launch_bounds__(kMatThreads) pairmatrix_kernel(const float* __restrict__ soa, int n, int n_pad,
+                                                                 int rb, int re, float cexp,
+                                                                 float* __restrict__ out) {
+  const int j0 = blockIdx.x * kMatCols + threadIdx.x * 4;
+  const int r0 = rb + blockIdx.y * kMatRows;
+  float pc[D][4];
+#pragma unroll
+  for (int c = 0; c < D; ++c) {
+    const float4 v = *reinterpret_cast<const float4*>(soa + (long long)c * n_pad + j0);  // n_pad covers j0+3
+    pc[c][0] = v.x; pc[c][1] = v.y; pc[c][2] = v.z; pc[c][3] = v.w;
+  }
+  const int rend = min(re, r0 + kMatRows);
+  for (int i = r0; i < rend; ++i) {
+    float a[D];
+#pragma unroll
+    for (int c = 0; c < D; ++c) a[c] = __ldg(soa + (long long)c * n_pad + i);
+    float o[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      float s = 0.f;
+#pragma unroll
+      for (int c = 0; c < D; ++c) {
+        const float d = pc[c][q] - a[c];
+        s = fmaf(d, d, s);
+      }
+      if (KTYPE == 0) o[q] = ex2_approx(cexp * s);  // exp(-gamma s) = 2^(-gamma log2(e) s)
+      else if (KTYPE == 1) o[q] = s;
+      else o[q] = sqrt_approx(s);
+    }
+    float* row = out + (size_t)(i - rb) * (size_t)n;
+    if (VEC) {
+      if (j0 < n) st_cs_v4(row + j0, o[0], o[1], o[2], o[3]);
+    } else {
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        if (j0 + q < n) __stcs(row + j0 + q, o[q]);
+    }
+  }
+}
+
+}  // namespace tbs

@@ -1,0 +1,38 @@
+"""Acceptance rules for GPU-vs-oracle parity (BASELINE.json north star)."""
+import numpy as np
+
+
+def check_sdh_float(h_gpu, h_or, amb):
+    """Float SDH: mass equal exactly; for every edge e, the cumulative counts
+    C(e) = sum_{b<e} h[b] differ by at most A_e (pairs within 1e-6 e w of edge e —
+    only those can change side under fp32 rounding). Implies per-bucket
+    |h_gpu[b] - h_or[b]| <= A_b + A_{b+1}. Returns diagnostics."""
+    g = np.asarray(h_gpu, dtype=np.int64)
+    o = np.asarray(h_or, dtype=np.int64)
+    a = np.asarray(amb, dtype=np.int64)
+    nb = len(o)
+    assert g.shape == o.shape
+    assert g.sum() == o.sum(), f"mass {g.sum()} != {o.sum()}"
+    cg, co = np.cumsum(g)[:-1], np.cumsum(o)[:-1]          # C(e) for e = 1..nb-1
+    dev = np.abs(cg - co)
+    bad = np.nonzero(dev > a[1:nb])[0]
+    assert bad.size == 0, f"edges {bad[:10] + 1}: |dC| {dev[bad[:10]]} > A_e {a[1:nb][bad[:10]]}"
+    per = np.abs(g - o)
+    lim = a[:nb] + a[1:nb + 1]
+    assert np.all(per <= lim)
+    return dict(max_bucket_diff=int(per.max()), edges_differing=int((dev > 0).sum()), amb_total=int(a.sum()))
+
+
+def check_pcf_float(c_gpu, c_or, amb):
+    assert abs(int(c_gpu) - int(c_or)) <= int(amb), f"{c_gpu} vs {c_or} (amb {amb})"
+
+
+def check_matrix(out_gpu, out_or, rtol=1e-5):
+    g = np.asarray(out_gpu, dtype=np.float64)
+    o = np.asarray(out_or, dtype=np.float64)
+    assert g.shape == o.shape
+    tiny = np.abs(o) < 1e-30
+    rel = np.where(tiny, np.abs(g - o) / 1e-30, np.abs(g - o) / np.where(tiny, 1.0, np.abs(o)))
+    m = float(rel.max()) if rel.size else 0.0
+    assert m <= rtol, f"max rel err {m}"
+    return m

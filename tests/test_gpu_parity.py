@@ -1,0 +1,225 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Acceptance (BASELINE.json north star):
+  * lattice SDH / 2PCF: bit-exact;
+  * float SDH: mass exact, cumulative counts within the edge-ambiguity counts A_e;
+  * float 2PCF: within A_r;
+  * Type-III: max relative error <= 1e-5.
+Small cases span several tiles (anchor tile 2048, partner chunk 1024) and ragged
+tails; full BASELINE.json sizes are checked in the bench's launch configuration on
+sampled anchor strips (the oracle computes them row by row) and on exact lattice
+closed forms.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import tbs_inputs as g
+from parity import check_matrix, check_pcf_float, check_sdh_float
+
+pytestmark = pytest.mark.gpu
+
+
+def dev(p):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(p)).cuda()
+
+
+def sdh_gpu(tbs, p, w, nb, **kw):
+    import torch
+    h = tbs.sdh(dev(p), w, nb, **kw)
+    torch.cuda.synchronize()
+    return h.cpu().numpy().astype(np.uint64)
+
+
+def w_of(nb, dim=3):
+    return float(np.float32(math.sqrt(dim) / nb))
+
+
+# ------------------------------------------------------------------ SDH float
+@pytest.mark.parametrize("n", [2, 3, 5, 100, 1023, 1024, 1025, 2047, 2048, 2049, 3071, 4096, 5000, 10007])
+def test_sdh_uniform_ragged(tbs, n):
+    p = g.uniform(n, 100 + n)
+    nb = 64
+    h = sdh_gpu(tbs, p, w_of(nb), nb)
+    ho, amb = oracle.sdh(p, w_of(nb), nb)
+    check_sdh_float(h, ho, amb)
+
+
+def test_sdh_config1(tbs):
+    """BASELINE.json configs[0]: N=4096 uniform, 64 buckets (golden from tools/make_goldens.py)."""
+    import json, os
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "sdh_uniform_n4096_nb64_seed1.json")))
+    p = g.uniform(4096, 1)
+    h = sdh_gpu(tbs, p, gold["w"], 64)
+    d = check_sdh_float(h, gold["hist"], gold["amb"])
+    assert int(h.sum()) == 8386560
+    print(d)
+
+
+@pytest.mark.parametrize("kind,nb", [("clustered", 256), ("uniform", 1000), ("uniform", 16384), ("clustered", 3)])
+def test_sdh_float_nb(tbs, kind, nb):
+    p = g.make(kind, 6000, 7)
+    h = sdh_gpu(tbs, p, w_of(nb), nb)
+    ho, amb = oracle.sdh(p, w_of(nb), nb)
+    check_sdh_float(h, ho, amb)
+
+
+@pytest.mark.parametrize("mode", ["lane", "cta", "global"])
+def test_sdh_hist_modes_float(tbs, mode):
+    p = g.clustered(5000, 9)
+    h = sdh_gpu(tbs, p, w_of(256), 256, hist_mode=mode)
+    ho, amb = oracle.sdh(p, w_of(256), 256)
+    check_sdh_float(h, ho, amb)
+
+
+@pytest.mark.parametrize("dim", [1, 2, 4])
+def test_sdh_dims(tbs, dim):
+    p = g.uniform(3000, 50 + dim, dim)
+    w = w_of(128, dim)
+    h = sdh_gpu(tbs, p, w, 128)
+    ho, amb = oracle.sdh(p, w, 128)
+    check_sdh_float(h, ho, amb)
+
+
+def test_sdh_offset_coordinates(tbs):
+    """Coordinates far from the origin: the kernel subtracts before it squares, so the
+    fp32 error stays relative to the distance (DESIGN.md §Error budget)."""
+    p = g.uniform(4000, 3) + np.float32(1000.0)
+    h = sdh_gpu(tbs, p, w_of(256), 256)
+    ho, amb = oracle.sdh(p, w_of(256), 256)
+    check_sdh_float(h, ho, amb)
+
+
+def test_sdh_all_coincident(tbs):
+    p = np.full((3000, 3), 0.3, np.float32)
+    h = sdh_gpu(tbs, p, 0.01, 16)
+    assert h[0] == 3000 * 2999 // 2 and h[1:].sum() == 0
+
+
+@pytest.mark.parametrize("n", [0, 1])
+def test_sdh_degenerate(tbs, n):
+    import torch
+    p = torch.zeros((n, 3), dtype=torch.float32, device="cuda")
+    h = tbs.sdh(p, 0.1, 8)
+    assert h.cpu().tolist() == [0] * 8
+
+
+# ------------------------------------------------------------------ SDH lattice (bit-exact)
+@pytest.mark.parametrize("n", [2, 17, 1500, 2048, 2049, 4096, 6001, 13824])
+def test_sdh_lattice_exact(tbs, n):
+    p = g.lattice(24, 5)[:n]
+    for (w, nb) in [(1.0, 64), (0.5, 80), (0.75, 7)]:
+        m, j = (1, 0) if w == 1.0 else ((1, 1) if w == 0.5 else (3, 2))
+        h = sdh_gpu(tbs, p, w, nb, lattice=True)
+        assert h.tolist() == oracle.sdh_lattice(p, m, j, nb).tolist(), (n, w, nb)
+
+
+@pytest.mark.parametrize("mode", [None, "lane", "cta", "global"])
+def test_sdh_lattice_modes_config1(tbs, mode):
+    """L=16 lattice (N=4096, the configs[0] size), w=2^-1, 64 buckets: closed form."""
+    p = g.lattice(16, 1)
+    h = sdh_gpu(tbs, p, 0.5, 64, lattice=True, hist_mode=mode)
+    assert h.tolist() == oracle.lattice_closed(16, 1, 1, 64)[0].tolist()
+    assert h.tolist() == oracle.sdh_lattice(p, 1, 1, 64).tolist()
+
+
+def test_sdh_lattice_float_mode_agrees(tbs):
+    """Float mode on a lattice with a dyadic width: exact except for pairs whose
+    distance is (numerically) on an edge — still inside the A_e rule."""
+    p = g.lattice(20, 2)
+    h = sdh_gpu(tbs, p, 0.5, 64)
+    ho, amb = oracle.sdh(p, 0.5, 64)
+    check_sdh_float(h, ho, amb)
+
+
+# ------------------------------------------------------------------ row ranges / multi-GPU partition
+@pytest.mark.parametrize("rows", [(0, 1), (1, 2), (5, 3000), (2047, 2049), (2048, 4096), (4000, 6000), (5999, 6000)])
+def test_sdh_row_ranges(tbs, rows):
+    p = g.lattice(20, 11)[:6000]
+    h = sdh_gpu(tbs, p, 1.0, 40, lattice=True, rows=rows)
+    assert h.tolist() == oracle.sdh_lattice(p, 1, 0, 40, rows=rows).tolist()
+
+
+@pytest.mark.parametrize("world", [2, 3, 4, 8])
+def test_partition_sums_bit_exact(tbs, world):
+    """Sum over the W rank strips (what all_reduce computes) == the W=1 result, bit-exact."""
+    import torch
+    p = dev(g.clustered(9000, 4))
+    full = tbs.sdh(p, w_of(256), 256).cpu()
+    acc = torch.zeros(256, dtype=torch.int64)
+    cacc = 0
+    for r in range(world):
+        rows = tbs.rank_rows(9000, world, r)
+        acc += tbs.sdh(p, w_of(256), 256, rows=rows).cpu()
+        cacc += int(tbs.pcf(p, 0.03, rows=rows).item())
+    assert torch.equal(acc, full)
+    assert cacc == int(tbs.pcf(p, 0.03).item())
+
+
+# ------------------------------------------------------------------ 2PCF
+@pytest.mark.parametrize("n", [2, 999, 2048, 4097, 13824])
+def test_pcf_lattice_exact(tbs, n):
+    p = g.lattice(24, 3)[:n]
+    for r in (1.0, 3.0, 10.0, 40.0):
+        c = int(tbs.pcf(dev(p), r).item())
+        assert c == oracle.pcf(p, r)[0], (n, r)
+
+
+def test_pcf_clustered_float(tbs):
+    p = g.clustered(20000, 3)
+    for r in (0.0, 0.01, 0.03, 0.2):
+        c = int(tbs.pcf(dev(p), r).item())
+        co, amb = oracle.pcf(p, r)
+        check_pcf_float(c, co, amb)
+
+
+def test_pcf_equals_cumulative_sdh_lattice(tbs):
+    p = dev(g.lattice(18, 6))
+    h = tbs.sdh(p, 1.0, 30, lattice=True).cpu().numpy()
+    for e in (1, 5, 17):
+        assert int(tbs.pcf(p, float(e)).item()) == int(h[:e].sum())
+
+
+@pytest.mark.parametrize("dim", [1, 2, 4])
+def test_pcf_dims(tbs, dim):
+    p = g.uniform(3000, 60 + dim, dim)
+    c = int(tbs.pcf(dev(p), 0.1).item())
+    co, amb = oracle.pcf(p, 0.1)
+    check_pcf_float(c, co, amb)
+
+
+# ------------------------------------------------------------------ Type-III
+@pytest.mark.parametrize("n", [1, 5, 1000, 1027, 2048, 3001])
+@pytest.mark.parametrize("kernel", ["gaussian", "dist2", "dist"])
+def test_pairmatrix(tbs, n, kernel):
+    p = g.uniform(n, 200 + n)
+    out = tbs.pairmatrix(dev(p), 1.0, kernel=kernel).cpu().numpy()
+    ref = oracle.pairmatrix(p, 1.0, ktype=tbs.KERNELS[kernel])
+    check_matrix(out, ref)
+    if kernel == "gaussian":
+        assert np.all(np.diag(out) == 1.0)
+
+
+def test_pairmatrix_rows_gamma(tbs):
+    p = g.uniform(2500, 8)
+    out = tbs.pairmatrix(dev(p), 3.5, rows=(700, 1333)).cpu().numpy()
+    check_matrix(out, oracle.pairmatrix(p, 3.5, rows=(700, 1333)))
+
+
+# ------------------------------------------------------------------ host-pointer ABI
+def test_host_pointer_entry_points(tbs):
+    p = g.clustered(7000, 5)
+    h = tbs.sdh_host(p, w_of(256), 256)
+    assert h.tolist() == sdh_gpu(tbs, p, w_of(256), 256).tolist()
+    assert tbs.pcf_host(p, 0.02) == int(tbs.pcf(dev(p), 0.02).item())
+    q = p[:700]
+    np.testing.assert_array_equal(tbs.pairmatrix_host(q, 2.0), tbs.pairmatrix(dev(q), 2.0).cpu().numpy())
+
+
+def test_launch_counter_moves(tbs):
+    before = tbs.launch_count()
+    sdh_gpu(tbs, g.uniform(3000, 1), 0.05, 32)
+    assert tbs.launch_count() >= before + 2           # loader + pair kernel
