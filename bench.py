@@ -1,0 +1,370 @@
+"""bench.py — throughput of the 2-BS hot path on B200 (one JSON line on rank 0).
+
+Default workload (BASELINE.json configs[1], the metric's N=1M point): SDH of
+N = 2^20 uniform 3-D points, 256 buckets, w = fp32(sqrt(3)/256). One step = one
+full pass of the hot path: SoA loader -> triangular pair kernel with the privatised
+shared-memory histogram -> u64 flush (-> NCCL all_reduce of the histogram for N>1).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NAME] [--impl tbs|reference]
+
+Multi-GPU: launched by torchrun, one rank per GPU; each rank computes its
+pair-balanced anchor strip (tbs_rank_rows) and the ranks sum their histograms with
+one all_reduce (strong scaling: the problem is fixed). Time = CUDA events on the
+launching stream around exactly K steps, barrier + synchronize on both sides, max
+over ranks. The L2 (126 MB) is flushed between steps by writing 256 MiB; the
+inputs (12 MiB) are smaller than L2 and the flush is inside the timed region.
+--impl reference times the CPU oracle (the reference arm of this tier) on bounded
+samples of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import tbs_inputs as gen  # noqa: E402
+
+WORKLOADS = {
+    # name: (op, distribution, n, seed, params)
+    "sdh_uniform_1m": ("sdh", "uniform", 1 << 20, 2, dict(nb=256)),         # configs[1] (default)
+    "sdh_clustered_1m": ("sdh", "clustered", 1 << 20, 3, dict(nb=256)),
+    "sdh_uniform_4m": ("sdh", "uniform", 1 << 22, 6, dict(nb=256)),         # north-star target line
+    "sdh_uniform_2m_16k": ("sdh", "uniform", 1 << 21, 4, dict(nb=16384)),   # configs[3]
+    "sdh_lattice_4m": ("sdh_lattice", "lattice", 160 ** 3, 6, dict(nb=256, w=1.0)),
+    "pcf_clustered_4m": ("pcf", "clustered", 1 << 22, 3, dict(r=0.03)),     # configs[2]
+    "pairmatrix_64k": ("pairmatrix", "uniform", 1 << 16, 5, dict(gamma=1.0)),  # configs[4]
+}
+METRIC = "SDH pair-distances/sec (G pairs/s) at N=1M–4M, 1/2/4/8 B200, % of roofline"
+
+# Roofline denominators: B200 unit counts x max SM clock.
+SMS = 148
+FP32_LANES_PER_CLK_SM = 128        # FFMA/FADD lanes per SM per clock (FFMA2 issues half as often, same lanes)
+ATOMS_LANES_PER_CLK_SM = 16        # shared-memory atomic lanes per SM per clock (measured 14.8, tools/peaks.cu)
+
+
+def peaks():
+    mp = {}
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            mp = json.load(f)
+    f_max = float(mp.get("sm_max_mhz", 1965.0)) * 1e6
+    return dict(
+        f_max=f_max,
+        fp32=SMS * FP32_LANES_PER_CLK_SM * f_max,
+        atoms=SMS * ATOMS_LANES_PER_CLK_SM * f_max,
+        hbm=float(mp.get("hbm_gbs", 6650.0)) * 1e9,
+        hbm_src="MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in mp else "fallback 6.65 TB/s (B200_PROFILING.md)",
+    )
+
+
+def units_of(op, n):
+    return n * n if op == "pairmatrix" else n * (n - 1) // 2
+
+
+# ------------------------------------------------------------------ clocks sampler
+class Clocks:
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.p = None
+        self.out = os.path.join("/tmp", f"tbs_clocks_{os.getpid()}.csv")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                       "-i", str(gpu_index), "-lms", "100"], stdout=open(self.out, "w"),
+                                      stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        self.p.wait()
+        rows = []
+        for line in open(self.out):
+            f = [x.strip() for x in line.split(",")]
+            if len(f) >= 7:
+                try:
+                    rows.append((float(f[0]), float(f[1]), f[3:7]))
+                except ValueError:
+                    pass
+        if not rows:
+            return None
+        load = [r for r in rows if r[0] > 500] or rows
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in load for i, v in enumerate(r[2]) if v.lower().startswith("active")})
+        return {"sm_mhz": statistics.median(r[0] for r in load), "sm_max_mhz": max(r[1] for r in rows),
+                "reasons": reasons, "samples": len(load)}
+
+
+# ------------------------------------------------------------------ reference arm (CPU oracle)
+def oracle_rate(op, p, params, rows):
+    import oracle
+    n = p.shape[0]
+    t0 = time.perf_counter()
+    if op == "sdh":
+        oracle.sdh(p, float(np.float32(math.sqrt(3) / params["nb"])), params["nb"], rows=rows)
+    elif op == "sdh_lattice":
+        oracle.sdh_lattice(p, 1, 0, params["nb"], rows=rows)
+    elif op == "pcf":
+        oracle.pcf(p, params["r"], rows=rows)
+    else:
+        oracle.pairmatrix(p, params["gamma"], rows=rows)
+    dt = time.perf_counter() - t0
+    b, e = rows
+    units = (e - b) * n if op == "pairmatrix" else (e - b) * (2 * n - b - e - 1) // 2
+    return units, dt
+
+
+def sample_rows(op, n, target_units):
+    """Anchor rows [0, R) holding about target_units pairs (matrix: entries)."""
+    per = n if op == "pairmatrix" else max(n - 1, 1)
+    return (0, int(min(n, max(1, target_units // per))))
+
+
+def cpu_baseline(op, p, params, seconds):
+    import oracle
+    n = p.shape[0]
+    u, dt = oracle_rate(op, p, params, sample_rows(op, n, 2e8 if op != "pairmatrix" else 2e7))
+    rate = u / dt
+    rows = sample_rows(op, n, rate * seconds)
+    u, dt = oracle_rate(op, p, params, rows)
+    return dict(value=u / dt / 1e9, unit="G pairs/s" if op != "pairmatrix" else "G entries/s",
+                cores=oracle.num_threads(), kind="oracle",
+                sample=f"anchor rows [{rows[0]},{rows[1]}) of the same N={n} input ({u:.3e} "
+                       f"{'pairs' if op != 'pairmatrix' else 'entries'}, {dt:.1f} s, fp64, OpenMP)")
+
+
+def run_reference(args, wl):
+    op, dist_, n, seed, params = WORKLOADS[wl]
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    p = gen.make(dist_, n, seed)
+    unit = "G pairs/s" if op != "pairmatrix" else "G entries/s"
+    import oracle
+    # each step: a bounded anchor-row sample, sized for ~120 s over the whole run
+    per_step = max(2.0, 120.0 / max(1, args.steps + args.warmup))
+    u0, dt0 = oracle_rate(op, p, params, sample_rows(op, n, 2e8 if op != "pairmatrix" else 2e7))
+    rows = sample_rows(op, n, u0 / dt0 * per_step)
+    for _ in range(args.warmup):
+        oracle_rate(op, p, params, rows)
+    tot_u, tot_t = 0, 0.0
+    for _ in range(args.steps):
+        u, dt = oracle_rate(op, p, params, rows)
+        tot_u += u
+        tot_t += dt
+    v = tot_u / tot_t / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": unit, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_t / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": wl, "n": n, "distribution": dist_, "seed": seed, **params},
+            "cpu_baseline": {"value": v, "unit": unit, "cores": oracle.num_threads(), "kind": "oracle",
+                             "sample": f"per step anchor rows [{rows[0]},{rows[1]}) of the N={n} input"},
+            "e2e": {"value": v, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ GPU arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="sdh_uniform_1m", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="tbs", choices=["tbs", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    args = ap.parse_args()
+    assert args.warmup >= 3 or args.impl == "reference", "timing rules: >= 3 warm-up steps"
+    wl = args.workload
+    if args.impl == "reference":
+        return run_reference(args, wl)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_pitaksirianannt16_b200 as tbs
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    pg = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+        pg = dist.group.WORLD
+
+    op, dist_, n, seed, params = WORKLOADS[wl]
+    p_host = gen.make(dist_, n, seed)
+    pts = torch.from_numpy(p_host).to(dev)
+    st = torch.cuda.current_stream(dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    nb = params.get("nb", 1)
+    w = float(np.float32(math.sqrt(3) / nb)) if op == "sdh" else params.get("w", 1.0)
+    out = None
+    if op in ("sdh", "sdh_lattice"):
+        out = torch.empty(nb, dtype=torch.int64, device=dev)
+    elif op == "pcf":
+        out = torch.empty(1, dtype=torch.int64, device=dev)
+    else:
+        rows_pm = (n * rank // world, n * (rank + 1) // world)
+        out = torch.empty((rows_pm[1] - rows_pm[0], n), dtype=torch.float32, device=dev)
+
+    def step(events=None):
+        if op == "sdh":
+            tbs.sdh(pts, w, nb, out=out, events=events, group=pg)
+        elif op == "sdh_lattice":
+            tbs.sdh(pts, w, nb, lattice=True, out=out, events=events, group=pg)
+        elif op == "pcf":
+            tbs.pcf(pts, params["r"], out=out, events=events, group=pg)
+        else:
+            tbs.pairmatrix(pts, params["gamma"], out=out, events=events, group=pg)
+
+    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    for a, b in kev:            # materialise the cudaEvent_t handles passed through the C ABI
+        a.record(st)
+        b.record(st)
+    for _ in range(args.warmup):
+        flush.fill_(1)
+        step()
+    torch.cuda.synchronize(dev)
+    if pg is not None:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    clocks = Clocks(local) if rank == 0 else None
+    l0 = tbs.launch_count()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t0.record(st)
+    for k in range(args.steps):
+        flush.fill_(k & 0xFF)    # L2 flush between steps (256 MiB > 126 MB L2)
+        step(events=kev[k])
+    t1.record(st)
+    torch.cuda.synchronize(dev)
+    if pg is not None:
+        dist.barrier()
+    launches = tbs.launch_count() - l0
+    ck = clocks.stop() if clocks else None
+    ms = t0.elapsed_time(t1)
+    kms = [a.elapsed_time(b) for a, b in kev]
+    if pg is not None:
+        tt = torch.tensor([ms, sum(kms) / len(kms)], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms, kavg = tt.tolist()
+    else:
+        kavg = sum(kms) / len(kms)
+
+    units = units_of("pairmatrix" if op == "pairmatrix" else "sdh", n)
+    value = units * args.steps / (ms * 1e-3) / 1e9
+    unit = "G pairs/s" if op != "pairmatrix" else "G entries/s"
+    pk = peaks()
+    # dominant kernel (pair kernel / matrix kernel) on this rank: its share of the units
+    if op == "pairmatrix":
+        rows_pm = (n * rank // world, n * (rank + 1) // world)
+        rank_units = (rows_pm[1] - rows_pm[0]) * n
+        bytes_ = rank_units * 4.0
+        achieved = bytes_ / (kavg * 1e-3)
+        roof = {"bound": "hbm", "achieved": achieved / 1e9, "peak": pk["hbm"] / 1e9, "unit": "GB/s",
+                "frac": achieved / pk["hbm"], "peak_source": pk["hbm_src"],
+                "algorithmic_bytes_per_launch": bytes_}
+    else:
+        rb, re = tbs.rank_rows(n, world, rank)
+        rank_units = (re - rb) * (2 * n - rb - re - 1) // 2
+        pairs_s = rank_units / (kavg * 1e-3)
+        if op == "pcf":
+            peak = pk["fp32"] / 6
+            bound_note = "FP32 pipe: 6 lane-ops/pair (3 sub + 3 mul/fma)"
+        else:
+            peak = min(pk["fp32"] / 6, pk["atoms"])
+            bound_note = "min(FP32 pipe / 6 lane-ops per pair, shared-atomic lanes / 1 per pair)"
+        roof = {"bound": "alu", "achieved": pairs_s / 1e9, "peak": peak / 1e9, "unit": "G pairs/s",
+                "frac": pairs_s / peak, "peak_source": f"{bound_note}; 148 SMs x unit lanes/clk x "
+                                                      f"{pk['f_max'] / 1e6:.0f} MHz (DESIGN.md §Roofline)",
+                "frac_fp32": pairs_s * 6 / pk["fp32"]}
+    roof["traffic"] = None
+    prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(prof):
+        try:
+            roof["traffic"] = json.load(open(prof)).get(wl)
+        except Exception:
+            pass
+    roof["kernel_ms_avg"] = kavg
+
+    # e2e: host buffers through the public API, H2D of the points and D2H of the result each step
+    e2e = None
+    if op in ("sdh", "pcf"):
+        ph = torch.from_numpy(p_host).pin_memory()
+        if world == 1:
+            hh = np.zeros(nb if op == "sdh" else 1, np.uint64)
+
+            def e2e_step():
+                if op == "sdh":
+                    tbs.sdh_host(ph.numpy(), w, nb, out=hh)
+                else:
+                    tbs.pcf_host(ph.numpy(), params["r"])
+        else:
+            res_h = torch.empty(out.shape, dtype=out.dtype).pin_memory()
+
+            def e2e_step():
+                d = ph.to(dev, non_blocking=True)
+                if op == "sdh":
+                    r = tbs.sdh(d, w, nb, group=pg)
+                else:
+                    r = tbs.pcf(d, params["r"], group=pg)
+                res_h.copy_(r)
+        for _ in range(2):
+            e2e_step()
+        torch.cuda.synchronize(dev)
+        if pg is not None:
+            dist.barrier()
+        ke = max(2, args.steps // 2)
+        tw = time.perf_counter()
+        for _ in range(ke):
+            e2e_step()
+        torch.cuda.synchronize(dev)
+        te = time.perf_counter() - tw
+        if pg is not None:
+            tt = torch.tensor([te], dtype=torch.float64, device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            te = tt.item()
+        e2e = {"value": units * ke / te / 1e9, "unit": unit, "h2d_bytes_per_step": int(p_host.nbytes),
+               "d2h_bytes_per_step": int(out.numel() * 8)}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(op if op != "sdh_lattice" else "sdh_lattice", p_host, params, args.cpu_seconds)
+
+    if rank == 0:
+        cfg = {"workload": wl, "n": n, "distribution": dist_, "seed": seed, **params,
+               "l2": "flushed between steps (256 MiB write inside the timed region; inputs 12 B/point < L2)",
+               "parallelism": f"rows{world}" if world > 1 else "single",
+               "step": "loader + pair kernel + flush" + (" + all_reduce" if world > 1 and op != "pairmatrix" else "")}
+        if op == "sdh":
+            cfg["bucket_width"] = w
+        line = {"metric": METRIC if op in ("sdh", "sdh_lattice") else f"{op} throughput ({unit})",
+                "value": value, "unit": unit, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": "f32", "data": "synthetic", "config": cfg,
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
+                "clocks": ck}
+        print(json.dumps(line), flush=True)
+    if pg is not None:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
