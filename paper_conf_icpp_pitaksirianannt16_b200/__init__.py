@@ -21,7 +21,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libtbs.so")
+LIB_PATH = os.environ.get("TBS_LIB_VARIANT") or os.path.join(_HERE, "libtbs.so")  # variant: A/B experiments only
 
 TBS_OK, TBS_EINVAL, TBS_ENOMEM, TBS_ECUDA, TBS_EUNSUPPORTED = range(5)
 TBS_EXACT_LATTICE = 0x1

@@ -14,21 +14,24 @@ FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std
          "-Xcompiler", "-fPIC", "-shared", "-cudart", "static", "-Xptxas", "-v"]
 
 
-def build(force=False, verbose=False):
-    if not force and os.path.exists(LIB) and all(os.path.getmtime(LIB) >= os.path.getmtime(d) for d in DEPS):
-        return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC] + FLAGS + ["-I", os.path.join(ROOT, "include"), "-o", tmp] + SRCS
+def build(force=False, verbose=False, out=None, defines=()):
+    """Build libtbs.so (or, for A/B experiments, a variant at `out` with -D`defines`)."""
+    target = out or LIB
+    if not force and os.path.exists(target) and all(os.path.getmtime(target) >= os.path.getmtime(d) for d in DEPS):
+        return target
+    tmp = target + f".tmp{os.getpid()}"
+    cmd = [NVCC] + FLAGS + [f"-D{d}" for d in defines] + ["-I", os.path.join(ROOT, "include"), "-o", tmp] + SRCS
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
         raise RuntimeError("nvcc failed building libtbs.so")
-    with open(os.path.join(HERE, "csrc", "ptxas_report.txt"), "w") as f:
-        f.write(r.stderr)
+    if out is None:
+        with open(os.path.join(HERE, "csrc", "ptxas_report.txt"), "w") as f:
+            f.write(r.stderr)
     if verbose:
         sys.stderr.write(r.stderr)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":

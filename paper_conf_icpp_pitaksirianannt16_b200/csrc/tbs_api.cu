@@ -10,11 +10,48 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <type_traits>
 
 #include "tbs.h"
 #include "tbs_kernels.cuh"
 
 using namespace tbs;
+
+// Pair-engine configurations per output type: anchors/thread, partner chunk, CTAs/SM
+// (A/B-tunable with -D at build time, see tools/build_ab.py).
+#ifndef TBS_SDH_KA
+#define TBS_SDH_KA 4
+#endif
+#ifndef TBS_SDH_TP
+#define TBS_SDH_TP 512
+#endif
+#ifndef TBS_SDH_MINB
+#define TBS_SDH_MINB 4
+#endif
+#ifndef TBS_PCF_KA
+#define TBS_PCF_KA 8
+#endif
+#ifndef TBS_PCF_TP
+#define TBS_PCF_TP 1024
+#endif
+#ifndef TBS_PCF_MINB
+#define TBS_PCF_MINB 2
+#endif
+#ifndef TBS_LAT_KA
+#define TBS_LAT_KA 8
+#endif
+#ifndef TBS_LAT_TP
+#define TBS_LAT_TP 1024
+#endif
+#ifndef TBS_LAT_MINB
+#define TBS_LAT_MINB 2
+#endif
+#define TBS_SDH_CFG TBS_SDH_KA, TBS_SDH_TP, TBS_SDH_MINB
+#define TBS_PCF_CFG TBS_PCF_KA, TBS_PCF_TP, TBS_PCF_MINB
+#define TBS_LAT_CFG TBS_LAT_KA, TBS_LAT_TP, TBS_LAT_MINB
+using SdhCfg = Cfg<TBS_SDH_CFG>;
+using PcfCfg = Cfg<TBS_PCF_CFG>;
+using LatCfg = Cfg<TBS_LAT_CFG>;
 
 namespace {
 
@@ -64,12 +101,30 @@ int current_device(Device& d) {
   return TBS_OK;
 }
 
+Geom make_geom(int64_t n, int64_t rb, int64_t re, int ta, int tp) {
+  Geom g;
+  g.n = (int)n;
+  g.rb = (int)rb;
+  g.re = (int)re;
+  g.I0 = (int)(rb / ta);
+  g.I1 = (int)((re + ta - 1) / ta);
+  g.Mc = (int)((n + tp - 1) / tp);
+  g.ratio = ta / tp;
+  g.n_pad = (int)(((n + kPadAlign - 1) / kPadAlign) * kPadAlign);
+  const long long I0 = g.I0, I1 = g.I1;
+  g.items = (I1 - I0) * (long long)g.Mc - (long long)g.ratio * ((I1 * (I1 - 1) - I0 * (I0 - 1)) / 2);
+  return g;
+}
+
+int pad_rows(int64_t n) { return (int)(((n + kPadAlign - 1) / kPadAlign) * kPadAlign); }
+
 // Persistent grid for a pair-kernel instantiation: SMs x resident CTAs (at most one CTA per item).
-template <class Op, int D>
-int launch_pair(const Device& dev, const float* soa, const Geom& g, const Op& op, cudaStream_t st, cudaEvent_t eb,
-                cudaEvent_t ee) {
-  auto kern = pair_kernel<Op, D>;
-  const long long smem = ((op.smem_bytes() + 127) & ~127ll) + 2ll * D * kTP * 4 + 16;
+template <class Op, int D, class C>
+int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op& op, const uint32_t* bbox,
+                cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee) {
+  auto kern = pair_kernel<Op, D, C>;
+  const Geom g = make_geom(a->n, a->row_begin, a->row_end, C::TA, C::TP);
+  const long long smem = ((op.smem_bytes() + 127) & ~127ll) + 2ll * D * C::TP * 4 + 16;
   if (smem > dev.smem_optin) return fail(TBS_EUNSUPPORTED, "pair kernel needs %lld B smem > %d", smem, dev.smem_optin);
   TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
@@ -78,25 +133,11 @@ int launch_pair(const Device& dev, const float* soa, const Geom& g, const Op& op
   long long grid = (long long)dev.sms * occ;
   if (grid > g.items) grid = g.items;
   if (eb) TBS_CUDA(cudaEventRecord(eb, st));
-  kern<<<(unsigned)grid, kThreads, (size_t)smem, st>>>(soa, g, op);
+  kern<<<(unsigned)grid, kThreads, (size_t)smem, st>>>(soa, g, op, bbox);
   TBS_CUDA(cudaGetLastError());
   g_launches.fetch_add(1);
   if (ee) TBS_CUDA(cudaEventRecord(ee, st));
   return TBS_OK;
-}
-
-Geom make_geom(int64_t n, int64_t rb, int64_t re) {
-  Geom g;
-  g.n = (int)n;
-  g.rb = (int)rb;
-  g.re = (int)re;
-  g.I0 = (int)(rb / kTA);
-  g.I1 = (int)((re + kTA - 1) / kTA);
-  g.Mc = (int)((n + kTP - 1) / kTP);
-  g.n_pad = (int)(((n + kTA - 1) / kTA) * kTA);
-  const long long I0 = g.I0, I1 = g.I1;
-  g.items = (I1 - I0) * (long long)g.Mc - (long long)kRatio * ((I1 * (I1 - 1) - I0 * (I0 - 1)) / 2);
-  return g;
 }
 
 int validate_common(const tbs_args* a) {
@@ -111,13 +152,18 @@ int validate_common(const tbs_args* a) {
 }
 
 // SoA copy of the points in stream-ordered scratch; the loader also zeroes `zero` words.
+// The allocation holds SoA [D][n_pad] followed by the 2D+1 bounding-box words.
 int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long long* zero, long long zero_words,
-                cudaStream_t st) {
-  TBS_CUDA(cudaMallocAsync((void**)soa, (size_t)D * n_pad * sizeof(float), st));
+                cudaStream_t st, uint32_t** bbox) {
+  const size_t soa_bytes = (size_t)D * n_pad * sizeof(float);
+  TBS_CUDA(cudaMallocAsync((void**)soa, soa_bytes + 64, st));
+  *bbox = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(*soa) + soa_bytes);
+  TBS_CUDA(cudaMemsetAsync(*bbox, 0, 64, st));
   const int threads = 256;
   long long blocks = std::min<long long>((n_pad + threads - 1) / threads, 148ll * 16);
   blocks = std::max<long long>(blocks, 1);
-  soa_loader<<<(unsigned)blocks, threads, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, D, *soa, zero, zero_words);
+  soa_loader<<<(unsigned)blocks, threads, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, D, *soa, zero, zero_words,
+                                                   *bbox);
   TBS_CUDA(cudaGetLastError());
   g_launches.fetch_add(1);
   return TBS_OK;
@@ -142,9 +188,9 @@ struct SdhPlan {
 };
 
 template <int D, bool LAT>
-int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const Geom& g, float w, long long m, int j,
-                 int nb, unsigned long long* hist, unsigned long long* part, int G, cudaStream_t st, cudaEvent_t eb,
-                 cudaEvent_t ee) {
+int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const uint32_t* bbox, const tbs_args* g, float w,
+                 long long m, int j, int nb, unsigned long long* hist, unsigned long long* part, int G, cudaStream_t st,
+                 cudaEvent_t eb, cudaEvent_t ee) {
   if (pl.global) {
     SdhGlobalOp<LAT> op{};
     op.nb = nb;
@@ -154,29 +200,30 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const G
     op.sh = 2 * j;
     op.G = G;
     op.part = part;
-    int rc = launch_pair<SdhGlobalOp<LAT>, D>(dev, soa, g, op, st, eb, ee);
+    int rc = launch_pair<SdhGlobalOp<LAT>, D, SdhCfg>(dev, soa, g, op, bbox, st, eb, ee);
     if (rc) return rc;
     reduce_partials<<<(nb + 255) / 256, 256, 0, st>>>(part, G, nb, hist);
     TBS_CUDA(cudaGetLastError());
     g_launches.fetch_add(1);
     return TBS_OK;
   }
+  using C = typename std::conditional<LAT, LatCfg, SdhCfg>::type;
   auto fill = [&](auto& op, int R) {
     op.nb = nb;
-    op.rows = nb;
+    op.rows = LAT ? nb : nb + kGuard;
     op.inv_w = (float)(1.0 / (double)w);
     op.scale = (float)std::ldexp(1.0 / (double)m, j);
     op.m = (int)m;
     op.sh = 2 * j;
     op.hist = hist;
-    // per item, a replica receives at most (32/R) lanes x kWarps x kA x kTP increments
-    const long long per_item = (long long)(32 / R) * kWarps * kA * kTP;
+    // per item, a replica receives at most (32/R) lanes x kWarps x KA x TP increments
+    const long long per_item = (long long)(32 / R) * kWarps * C::KA * C::TP;
     op.flush_every = (int)std::max<long long>(1, (0xffffffffll / per_item) - 1);
   };
   switch (pl.log2r) {
-    case 5: { SdhSmemOp<5, LAT> op{}; fill(op, 32); return launch_pair<SdhSmemOp<5, LAT>, D>(dev, soa, g, op, st, eb, ee); }
-    case 2: { SdhSmemOp<2, LAT> op{}; fill(op, 4); return launch_pair<SdhSmemOp<2, LAT>, D>(dev, soa, g, op, st, eb, ee); }
-    default: { SdhSmemOp<0, LAT> op{}; fill(op, 1); return launch_pair<SdhSmemOp<0, LAT>, D>(dev, soa, g, op, st, eb, ee); }
+    case 5: { SdhSmemOp<5, LAT> op{}; fill(op, 32); return launch_pair<SdhSmemOp<5, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee); }
+    case 2: { SdhSmemOp<2, LAT> op{}; fill(op, 4); return launch_pair<SdhSmemOp<2, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee); }
+    default: { SdhSmemOp<0, LAT> op{}; fill(op, 1); return launch_pair<SdhSmemOp<0, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee); }
   }
 }
 
@@ -204,24 +251,24 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   // Output-stage plan: lane-private copies (R = 32) while they fit a 96 KB budget (two CTAs
   // per SM), then 4 replicas, then one copy per CTA; beyond that, global partial copies.
   SdhPlan pl{lattice, false, 5};
-  const long long part_budget = std::min<long long>(96 * 1024, dev.smem_optin - 2ll * 4 * kTP * 4 - 256);
-  const long long one_copy_budget = dev.smem_optin - 2ll * 4 * kTP * 4 - 256;
-  if ((long long)nb * 32 * 4 <= part_budget) pl.log2r = 5;
-  else if ((long long)nb * 4 * 4 <= part_budget) pl.log2r = 2;
-  else if ((long long)nb * 4 <= one_copy_budget) pl.log2r = 0;
+  const long long part_budget = std::min<long long>(96 * 1024, dev.smem_optin - 2ll * 4 * SdhCfg::TP * 4 - 256);
+  const long long one_copy_budget = dev.smem_optin - 2ll * 4 * SdhCfg::TP * 4 - 256;
+  if ((long long)(nb + kGuard) * 32 * 4 <= part_budget) pl.log2r = 5;
+  else if ((long long)(nb + kGuard) * 4 * 4 <= part_budget) pl.log2r = 2;
+  else if ((long long)(nb + kGuard) * 4 <= one_copy_budget) pl.log2r = 0;
   else pl.global = true;
   if (a->flags & TBS_HIST_FORCE_LANE) {
-    if ((long long)nb * 32 * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_LANE: nb too large for smem");
+    if ((long long)(nb + kGuard) * 32 * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_LANE: nb too large for smem");
     pl = SdhPlan{lattice, false, 5};
   }
   if (a->flags & TBS_HIST_FORCE_CTA) {
-    if ((long long)nb * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_CTA: nb too large for smem");
+    if ((long long)(nb + kGuard) * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_CTA: nb too large for smem");
     pl = SdhPlan{lattice, false, 0};
   }
   if (a->flags & TBS_HIST_FORCE_GLOBAL) pl = SdhPlan{lattice, true, 0};
 
   const int D = a->dim <= 3 ? 3 : 4;
-  const Geom g = make_geom(a->n, a->row_begin, a->row_end);
+  const int n_pad = pad_rows(a->n);
   int G = 0;
   unsigned long long* part = nullptr;
   long long zero_words = 0;
@@ -233,13 +280,15 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   float* soa = nullptr;
   // Smem modes accumulate into hist: the loader zeroes it. Global mode zeroes the partials
   // (the reduce kernel overwrites hist).
-  rc = load_points(a, D, g.n_pad, &soa, pl.global ? part : h, pl.global ? zero_words : nb, st);
+  uint32_t* bbox = nullptr;
+  rc = load_points(a, D, n_pad, &soa, pl.global ? part : h, pl.global ? zero_words : nb, st, &bbox);
+  if (a->flags & TBS_FORCE_CLAMP) bbox = nullptr;
   if (!rc) {
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
-    if (D == 3) rc = lattice ? sdh_dispatch<3, true>(dev, pl, soa, g, w, m, j, nb, h, part, G, st, eb, ee)
-                             : sdh_dispatch<3, false>(dev, pl, soa, g, w, m, j, nb, h, part, G, st, eb, ee);
-    else rc = lattice ? sdh_dispatch<4, true>(dev, pl, soa, g, w, m, j, nb, h, part, G, st, eb, ee)
-                      : sdh_dispatch<4, false>(dev, pl, soa, g, w, m, j, nb, h, part, G, st, eb, ee);
+    if (D == 3) rc = lattice ? sdh_dispatch<3, true>(dev, pl, soa, bbox, a, w, m, j, nb, h, part, G, st, eb, ee)
+                             : sdh_dispatch<3, false>(dev, pl, soa, bbox, a, w, m, j, nb, h, part, G, st, eb, ee);
+    else rc = lattice ? sdh_dispatch<4, true>(dev, pl, soa, bbox, a, w, m, j, nb, h, part, G, st, eb, ee)
+                      : sdh_dispatch<4, false>(dev, pl, soa, bbox, a, w, m, j, nb, h, part, G, st, eb, ee);
   }
   if (soa) cudaFreeAsync(soa, st);
   if (part) cudaFreeAsync(part, st);
@@ -260,15 +309,16 @@ int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
     return TBS_OK;
   }
   const int D = a->dim <= 3 ? 3 : 4;
-  const Geom g = make_geom(a->n, a->row_begin, a->row_end);
   float* soa = nullptr;
-  rc = load_points(a, D, g.n_pad, &soa, c, 1, st);
+  uint32_t* bbox = nullptr;
+  rc = load_points(a, D, pad_rows(a->n), &soa, c, 1, st, &bbox);
   if (!rc) {
     PcfOp op{};
     op.r2 = (float)((double)r * (double)r);
     op.count = c;
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
-    rc = D == 3 ? launch_pair<PcfOp, 3>(dev, soa, g, op, st, eb, ee) : launch_pair<PcfOp, 4>(dev, soa, g, op, st, eb, ee);
+    rc = D == 3 ? launch_pair<PcfOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee)
+                 : launch_pair<PcfOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee);
   }
   if (soa) cudaFreeAsync(soa, st);
   return rc;
@@ -300,9 +350,10 @@ int pairmatrix_impl(const tbs_args* a, tbs_kernel k, float* out) {
   if (a->row_end == a->row_begin || a->n == 0) return TBS_OK;
   cudaStream_t st = (cudaStream_t)a->stream;
   const int D = a->dim <= 3 ? 3 : 4;
-  const int n_pad = (int)(((a->n + kTA - 1) / kTA) * kTA);
+  const int n_pad = pad_rows(a->n);
   float* soa = nullptr;
-  rc = load_points(a, D, n_pad, &soa, nullptr, 0, st);
+  uint32_t* bbox = nullptr;
+  rc = load_points(a, D, n_pad, &soa, nullptr, 0, st, &bbox);
   if (!rc) {
     const float cexp = (float)(-(double)k.gamma * 1.4426950408889634);  // -gamma * log2(e)
     if (D == 3) rc = k.type == 0 ? matrix_launch<0, 3>(a, soa, n_pad, cexp, out, st)

@@ -6,7 +6,7 @@
 //   * SoA input (L338-341)                       -> loader writes [D][n_pad] fp32 SoA
 //   * block tiling, Alg. 2 (L366-458)            -> triangular (anchor tile, partner chunk)
 //                                                   work items over persistent CTAs
-//   * anchor datum in registers, Alg. 3 (L465-511)-> kA = 8 anchors per thread, packed in
+//   * anchor datum in registers, Alg. 3 (L465-511)-> KA anchors per thread (Cfg), packed in
 //                                                   f32x2 register pairs (FADD2/FFMA2)
 //   * partner block in cache (L499)              -> TMA bulk copy (cp.async.bulk) into
 //                                                   shared memory, double-buffered on mbarriers,
@@ -22,29 +22,43 @@
 
 namespace tbs {
 
+#ifndef TBS_PUNROLL
+#define TBS_PUNROLL 1                      // partner-quad loop unroll (software-pipelining freedom)
+#endif
+#ifndef TBS_ADDR_MODE
+#define TBS_ADDR_MODE 0                    // 0: LEA from the floor's bits; 1: FADD2 into a binade + IADD
+#endif
 constexpr int kThreads = 256;              // 8 warps per CTA
+constexpr int kPUnroll = TBS_PUNROLL;
 constexpr int kWarps = kThreads / 32;
-constexpr int kA = 8;                      // anchors per thread (4 f32x2 pairs)
-constexpr int kTA = kThreads * kA;         // anchor tile: 2048 points
-constexpr int kTP = 1024;                  // partner chunk: 1024 points
-constexpr int kRatio = kTA / kTP;          // partner chunks per anchor tile
+constexpr int kPadAlign = 2048;            // SoA rows padded to a multiple of every anchor tile / chunk
 constexpr uint32_t kMagic = 0x4B000000u;   // bits of 2^23: x + 2^23 (round-down) = 2^23 + floor(x)
 constexpr float kMagicF = 8388608.0f;
 constexpr int kNoAnchor = 0x7fffffff;      // masked anchor index (no partner is greater)
 
-// Work decomposition (host-computed). Anchor tiles I in [I0, I1) of kTA points; for each,
-// partner chunks J in [I*kRatio, Mc) of kTP points. Item count: sum_I (Mc - I*kRatio).
+// Pair-engine configuration: KA anchors per thread (register-blocked, packed in KA/2
+// f32x2 pairs), TP partners per staged chunk, MINB resident CTAs per SM that the
+// register budget targets. Anchor tile TA = 256 * KA points.
+template <int KA_, int TP_, int MINB_>
+struct Cfg {
+  static constexpr int KA = KA_, TP = TP_, MINB = MINB_, TA = kThreads * KA_, RATIO = TA / TP_;
+  static_assert(KA_ % 2 == 0 && TP_ % 4 == 0 && TA % TP_ == 0 && kPadAlign % TA == 0, "bad pair-engine config");
+};
+
+// Work decomposition (host-computed). Anchor tiles I in [I0, I1) of TA points; for each,
+// partner chunks J in [I*ratio, Mc) of TP points. Item count: sum_I (Mc - I*ratio).
 struct Geom {
   int n;            // number of points
   int rb, re;       // anchor rows [rb, re)
   int I0, I1;       // anchor tiles
-  int Mc;           // ceil(n / kTP)
-  int n_pad;        // SoA row stride (multiple of kTA)
+  int Mc;           // ceil(n / TP)
+  int ratio;        // TA / TP
+  int n_pad;        // SoA row stride (multiple of kPadAlign)
   long long items;  // total work items
 };
 
 __device__ __forceinline__ long long items_before(const Geom& g, long long I) {
-  return (I - g.I0) * (long long)g.Mc - (long long)kRatio * ((I * (I - 1) - (long long)g.I0 * (g.I0 - 1)) / 2);
+  return (I - g.I0) * (long long)g.Mc - (long long)g.ratio * ((I * (I - 1) - (long long)g.I0 * (g.I0 - 1)) / 2);
 }
 __device__ __forceinline__ void item_to_tile(const Geom& g, long long it, int& I, int& J) {
   int lo = g.I0, hi = g.I1 - 1;
@@ -53,22 +67,73 @@ __device__ __forceinline__ void item_to_tile(const Geom& g, long long it, int& I
     if (items_before(g, mid) <= it) lo = mid; else hi = mid - 1;
   }
   I = lo;
-  J = lo * kRatio + (int)(it - items_before(g, lo));
+  J = lo * g.ratio + (int)(it - items_before(g, lo));
 }
 
 // ------------------------------------------------------------------------------------
 // a1: SoA loader. AoS [n][dim] -> SoA [D][n_pad] (pad coordinates and pad points = 0).
 // Also zeroes `zero_words` u64 words at `zero` (the caller's output / partial copies),
-// saving a separate memset launch.
+// saving a separate memset launch, and reduces the bounding box of the points into
+// `bbox` (zero-initialised): bbox[c] = max of ~ord(x_c), bbox[D + c] = max of ord(x_c),
+// with ord() the order-preserving float -> u32 map; bbox[2D] |= 1 on a non-finite
+// coordinate. The pair kernel uses it to prove that no distance can leave the
+// histogram's guard rows, which lets it drop the clamp instruction.
 // ------------------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t f2ord(float x) {
+  const uint32_t b = __float_as_uint(x);
+  return (b & 0x80000000u) ? ~b : (b | 0x80000000u);
+}
+__device__ __forceinline__ float ord2f(uint32_t o) {
+  return __uint_as_float((o & 0x80000000u) ? (o & 0x7fffffffu) : ~o);
+}
+
 __global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_pad, int D,
-                           float* __restrict__ soa, unsigned long long* __restrict__ zero, long long zero_words) {
+                           float* __restrict__ soa, unsigned long long* __restrict__ zero, long long zero_words,
+                           uint32_t* __restrict__ bbox) {
   const long long stride = (long long)gridDim.x * blockDim.x;
+  uint32_t lo[4] = {0u, 0u, 0u, 0u}, hi[4] = {0u, 0u, 0u, 0u}, bad = 0u;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n_pad; i += stride) {
-    for (int c = 0; c < D; ++c)
-      soa[(long long)c * n_pad + i] = (i < n && c < dim) ? __ldg(pts + i * dim + c) : 0.0f;
+    for (int c = 0; c < D; ++c) {
+      float v = 0.0f;
+      if (i < n && c < dim) {
+        v = __ldg(pts + i * dim + c);
+        const uint32_t o = f2ord(v);
+        lo[c] = max(lo[c], ~o);
+        hi[c] = max(hi[c], o);
+        bad |= isfinite(v) ? 0u : 1u;
+      }
+      soa[(long long)c * n_pad + i] = v;
+    }
   }
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < zero_words; i += stride) zero[i] = 0ull;
+  if (bbox) {
+    for (int c = 0; c < D; ++c) {
+      uint32_t a = lo[c], b = hi[c];
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) {
+        a = max(a, __shfl_xor_sync(0xffffffffu, a, off));
+        b = max(b, __shfl_xor_sync(0xffffffffu, b, off));
+      }
+      if ((threadIdx.x & 31) == 0) {
+        if (a) atomicMax(bbox + c, a);
+        if (b) atomicMax(bbox + D + c, b);
+      }
+    }
+    bad = __any_sync(0xffffffffu, bad != 0u) ? 1u : 0u;
+    if ((threadIdx.x & 31) == 0 && bad) atomicOr(bbox + 2 * D, 1u);
+  }
+}
+
+// Upper bound on any pair distance from the loader's bounding box (+inf if unknown).
+__device__ __forceinline__ float bbox_diameter(const uint32_t* __restrict__ bbox, int D) {
+  if (bbox == nullptr || bbox[2 * D] != 0u) return __int_as_float(0x7f800000);
+  double s = 0.0;
+  for (int c = 0; c < D; ++c) {
+    if (bbox[c] == 0u || bbox[D + c] == 0u) return __int_as_float(0x7f800000);
+    const double e = (double)ord2f(bbox[D + c]) - (double)ord2f(~bbox[c]);
+    s += e * e;
+  }
+  return (float)(sqrt(s) * (1.0 + 1e-5));
 }
 
 // ------------------------------------------------------------------------------------
@@ -84,18 +149,35 @@ __global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_
 // Type-II, float mode: bucket = min(floor(sqrt(s) / w), nb - 1) with R replicas per bin
 // in shared memory, layout word[k * R + (lane & (R-1))]. R = 32: every lane owns a copy
 // and the 32 lanes of an ATOMS hit 32 distinct banks (no conflicts, no same-address).
+//
+// Address arithmetic on the FMA pipe, two pairs per instruction:
+//   y = RD(q * inv_w + 2^23)            FFMA2.RM: y = 2^23 + floor(q / w)       (exact)
+//   z = y + (lane_r / R - 2^23 + 2^E)   FADD2:    z = 2^E + k + lane_r / R       (exact)
+// with E = 21 - log2(R): in the binade [2^E, 2^(E+1)) one unit of k is 4R bytes of the
+// float's bit pattern, so bits(z) - bits(2^E) = 4 (k R + lane_r) is the byte offset of
+// the lane's counter. The remaining add of (smem base - bits(2^E)) is CTA-uniform and
+// folds into the ATOMS addressing mode ([R + UR]) — no integer instruction per pair.
+// The clamp k <= nb-1 (one FMNMX per pair) is dropped when the loader's bounding box
+// proves k < nb + kGuard for every pair; guard rows are folded into nb-1 at the flush.
 // LATTICE: exact integer bucketing max{k : (k m)^2 <= 4^j s} for integer-valued input.
+constexpr int kGuard = 32;
+
+extern __shared__ __align__(128) unsigned char tbs_smem[];  // dynamic smem; histogram at offset 0
+
 template <int LOG2R, bool LATTICE>
 struct SdhSmemOp {
   static constexpr int R = 1 << LOG2R;
+  static constexpr int E = 21 - LOG2R;
   int nb;             // buckets
-  int rows;           // rows allocated (= nb)
+  int rows;           // rows allocated (nb, + kGuard in float mode)
   float inv_w;        // fp32(1 / w)                       (float mode)
   float scale;        // fp32(2^j / m)                     (lattice mode)
   int m, sh;          // w = m * 2^-j, sh = 2 j            (lattice mode)
   unsigned long long* hist;  // global u64 output [nb]
-  uint32_t base;      // shared address of word 0 for this lane, minus the magic offset
-  uint32_t bmax;      // magic bits of bucket nb-1 (clamp)
+  uint32_t base;      // lattice: shared address of word 0 for this lane, minus the magic offset
+  uint32_t bmax;      // lattice: magic bits of bucket nb-1 (clamp)
+  float zc;           // float: lane_r / R - 2^23 + 2^E
+  float ymax;         // float: 2^23 + nb - 1
   int flush_every;    // items between overflow flushes
 
   __host__ __device__ long long smem_bytes() const { return (long long)rows * R * 4; }
@@ -103,45 +185,58 @@ struct SdhSmemOp {
   __device__ __forceinline__ void init(unsigned char* smem) {
     uint32_t* h = reinterpret_cast<uint32_t*>(smem);
     for (int i = threadIdx.x; i < rows * R; i += kThreads) h[i] = 0u;
-    const int lane = threadIdx.x & 31;
-    base = smem_addr(smem) + (uint32_t)((lane & (R - 1)) * 4) - (kMagic << (LOG2R + 2));
+    const int lane_r = threadIdx.x & (R - 1);
+    base = smem_addr(smem) + (uint32_t)(lane_r * 4) - (kMagic << (LOG2R + 2));
     bmax = kMagic + (uint32_t)(nb - 1);
+    zc = (float)lane_r / (float)R - (kMagicF - (float)(1 << E));
+    ymax = kMagicF + (float)(nb - 1);
   }
   __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
-
-  __device__ __forceinline__ uint32_t bucket_bits(float s) const {
-    if (!LATTICE) {
-      return 0u;  // unused (packed path below)
-    } else {
-      // s is an exact integer < 2^24. fp32 estimate, then exact integer fix-up by one step.
-      uint32_t si = __float2uint_rz(s);
-      float q = sqrt_approx(s);
-      int k = min((int)(__float_as_uint(__fmaf_rd(q, scale, kMagicF)) - kMagic), nb);
-      unsigned long long S = (unsigned long long)si << sh;
-      unsigned long long e1 = (unsigned long long)(k + 1) * (unsigned long long)m;
-      k += (e1 * e1 <= S) ? 1 : 0;
-      unsigned long long e0 = (unsigned long long)k * (unsigned long long)m;
-      k -= (e0 * e0 > S) ? 1 : 0;
-      return kMagic + (uint32_t)k;
-    }
+  __device__ __forceinline__ bool needs_clamp(const uint32_t* bbox, int D) const {
+    if (LATTICE) return true;
+    const float dmax = bbox_diameter(bbox, D);
+    return !(dmax * inv_w < (float)(nb + kGuard - 2));
   }
 
-  template <bool MASKED>
+  __device__ __forceinline__ uint32_t bucket_bits(float s) const {
+    // lattice: s is an exact integer < 2^24. fp32 estimate, then exact integer fix-up by one step.
+    uint32_t si = __float2uint_rz(s);
+    float q = sqrt_approx(s);
+    int k = min((int)(__float_as_uint(__fmaf_rd(q, scale, kMagicF)) - kMagic), nb);
+    unsigned long long S = (unsigned long long)si << sh;
+    unsigned long long e1 = (unsigned long long)(k + 1) * (unsigned long long)m;
+    k += (e1 * e1 <= S) ? 1 : 0;
+    unsigned long long e0 = (unsigned long long)k * (unsigned long long)m;
+    k -= (e0 * e0 > S) ? 1 : 0;
+    return kMagic + (uint32_t)k;
+  }
+
+  template <bool MASKED, bool CLAMP>
   __device__ __forceinline__ void pair2(float2 s, int pv, int a0, int a1) {
-    uint32_t b0, b1;
+    uint32_t ad0, ad1;
     if (!LATTICE) {
-      // floor(sqrt(s) * inv_w) via one FFMA2.RM onto 2^23: the scale and the floor in one op
-      float2 q = make_float2(sqrt_approx(s.x), sqrt_approx(s.y));
-      float2 k = __ffma2_rd(q, make_float2(inv_w, inv_w), make_float2(kMagicF, kMagicF));
-      b0 = __float_as_uint(k.x);
-      b1 = __float_as_uint(k.y);
+      const float2 q = make_float2(sqrt_approx(s.x), sqrt_approx(s.y));
+      float2 y = __ffma2_rd(q, make_float2(inv_w, inv_w), make_float2(kMagicF, kMagicF));
+      if (CLAMP) {
+        y.x = fminf(y.x, ymax);
+        y.y = fminf(y.y, ymax);
+      }
+#if TBS_ADDR_MODE == 1
+      const float2 z = __fadd2_rn(y, make_float2(zc, zc));
+      // uniform part recomputed from the smem symbol so ptxas may fold it into [R + UR]
+      const uint32_t ub = smem_addr(tbs_smem) - __float_as_uint((float)(1 << E));
+      ad0 = __float_as_uint(z.x) + ub;
+      ad1 = __float_as_uint(z.y) + ub;
+#else
+      // bits(y) = 2^23's bits + k: one shift-add (LEA) gives base + 4 (k R + lane_r)
+      ad0 = (__float_as_uint(y.x) << (LOG2R + 2)) + base;
+      ad1 = (__float_as_uint(y.y) << (LOG2R + 2)) + base;
+#endif
     } else {
-      b0 = bucket_bits(s.x);
-      b1 = bucket_bits(s.y);
+      const uint32_t b0 = min(bucket_bits(s.x), bmax), b1 = min(bucket_bits(s.y), bmax);
+      ad0 = (b0 << (LOG2R + 2)) + base;
+      ad1 = (b1 << (LOG2R + 2)) + base;
     }
-    b0 = min(b0, bmax);
-    b1 = min(b1, bmax);
-    const uint32_t ad0 = (b0 << (LOG2R + 2)) + base, ad1 = (b1 << (LOG2R + 2)) + base;
     if (MASKED) {
       red_smem_inc_gt(ad0, pv, a0);
       red_smem_inc_gt(ad1, pv, a1);
@@ -208,7 +303,8 @@ struct SdhGlobalOp {
     }
     return min(k, nb - 1);
   }
-  template <bool MASKED>
+  __device__ __forceinline__ bool needs_clamp(const uint32_t*, int) const { return false; }
+  template <bool MASKED, bool CLAMP>
   __device__ __forceinline__ void pair2(float2 s, int pv, int a0, int a1) {
     unsigned long long* p0 = mine + bucket(s.x);
     unsigned long long* p1 = mine + bucket(s.y);
@@ -229,13 +325,14 @@ struct SdhGlobalOp {
 struct PcfOp {
   float r2;
   unsigned long long* count;
-  uint32_t c;                // per-item counter (<= kA * kTP)
+  uint32_t c;                // per-item counter (<= KA * TP)
   unsigned long long total;  // per-thread running total
 
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) { c = 0u; total = 0ull; }
   __device__ __forceinline__ float2 bias() const { return make_float2(-r2, -r2); }
-  template <bool MASKED>
+  __device__ __forceinline__ bool needs_clamp(const uint32_t*, int) const { return false; }
+  template <bool MASKED, bool CLAMP>
   __device__ __forceinline__ void pair2(float2 t, int pv, int a0, int a1) {
     uint32_t s0 = __float_as_uint(t.x) >> 31, s1 = __float_as_uint(t.y) >> 31;
     if (MASKED) {
@@ -267,27 +364,39 @@ struct PcfOp {
 
 // ------------------------------------------------------------------------------------
 // a2-a10: the pair engine. Persistent CTAs walk a contiguous range of the linearised
-// triangular item list. Per item: anchors (kA per thread) in registers, partner chunk
+// triangular item list. Per item: anchors (KA per thread) in registers, partner chunk
 // staged by TMA into a double-buffered smem slot, every (anchor, partner) pair evaluated
 // as packed f32x2 arithmetic, the Op consumes the squared distances.
 // ------------------------------------------------------------------------------------
-template <class Op, int D>
+template <int D, int TP>
 __device__ __forceinline__ void issue_chunk(const float* __restrict__ soa, const Geom& g, int J, float* dst,
                                             uint32_t bar) {
-  mbar_arrive_expect_tx(bar, D * kTP * 4);
+  mbar_arrive_expect_tx(bar, D * TP * 4);
 #pragma unroll
   for (int c = 0; c < D; ++c)
-    bulk_g2s(smem_addr(dst + c * kTP), soa + (long long)c * g.n_pad + (long long)J * kTP, kTP * 4, bar);
+    bulk_g2s(smem_addr(dst + c * TP), soa + (long long)c * g.n_pad + (long long)J * TP, TP * 4, bar);
 }
 
-template <class Op, int D, bool MASKED>
-__device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, const float2 (&na)[D][kA / 2],
-                                          const int (&aidx)[kA], int p0, int cnt, int n) {
+template <class Op, int D, class C, bool MASKED, bool CLAMP>
+__device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, const float2 (&na)[D][C::KA / 2],
+                                          const Geom& g, int I, int p0, int cnt) {
+  // masked items only: anchor index or kNoAnchor outside [rb, re) (built here so the
+  // registers are not live in the unmasked loop)
+  int aidx[C::KA];
+  if (MASKED) {
+#pragma unroll
+    for (int k = 0; k < C::KA; ++k) {
+      const int a = I * C::TA + k * kThreads + (int)threadIdx.x;
+      aidx[k] = (a >= g.rb && a < g.re) ? a : kNoAnchor;
+    }
+  }
+  const int n = g.n;
+#pragma unroll kPUnroll
   for (int p = 0; p < cnt; p += 4) {
     float c4[D][4];
 #pragma unroll
     for (int c = 0; c < D; ++c) {
-      const float4 v = *reinterpret_cast<const float4*>(B + c * kTP + p);
+      const float4 v = *reinterpret_cast<const float4*>(B + c * C::TP + p);
       c4[c][0] = v.x; c4[c][1] = v.y; c4[c][2] = v.z; c4[c][3] = v.w;
     }
 #pragma unroll
@@ -295,7 +404,7 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
       int pv = 0;
       if (MASKED) pv = (p0 + p + q < n) ? p0 + p + q : -1;
 #pragma unroll
-      for (int m = 0; m < kA / 2; ++m) {
+      for (int m = 0; m < C::KA / 2; ++m) {
         float2 d = __fadd2_rn(na[0][m], make_float2(c4[0][q], c4[0][q]));
         float2 s = __ffma2_rn(d, d, op.bias());
 #pragma unroll
@@ -303,22 +412,24 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
           d = __fadd2_rn(na[c][m], make_float2(c4[c][q], c4[c][q]));
           s = __ffma2_rn(d, d, s);
         }
-        op.template pair2<MASKED>(s, pv, aidx[2 * m], aidx[2 * m + 1]);
+        op.template pair2<MASKED, CLAMP>(s, pv, MASKED ? aidx[2 * m] : 0, MASKED ? aidx[2 * m + 1] : 0);
       }
     }
   }
 }
 
-template <class Op, int D>
-__global__ void __launch_bounds__(kThreads, 2) pair_kernel(const float* __restrict__ soa, Geom g, Op op) {
-  extern __shared__ __align__(128) unsigned char smem[];
+template <class Op, int D, class C>
+__global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __restrict__ soa, Geom g, Op op,
+                                                            const uint32_t* __restrict__ bbox) {
+  unsigned char* smem = tbs_smem;
   const long long hbytes = (op.smem_bytes() + 127) & ~127ll;
   float* bufs = reinterpret_cast<float*>(smem + hbytes);
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + hbytes + 2 * D * kTP * 4);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + hbytes + 2 * D * C::TP * 4);
   const uint32_t bar0 = smem_addr(bars), bar1 = smem_addr(bars + 1);
   const int tid = threadIdx.x;
 
   op.init(smem);
+  const bool clamp = op.needs_clamp(bbox, D);
   if (tid == 0) {
     mbar_init(bar0, 1);
     mbar_init(bar1, 1);
@@ -331,23 +442,21 @@ __global__ void __launch_bounds__(kThreads, 2) pair_kernel(const float* __restri
   if (beg < end) {
     int I, J;
     item_to_tile(g, beg, I, J);
-    if (tid == 0) issue_chunk<Op, D>(soa, g, J, bufs, bar0);
+    if (tid == 0) issue_chunk<D, C::TP>(soa, g, J, bufs, bar0);
     int curI = -1;
     uint32_t phase = 0u;  // bit s = parity of buffer s
     int since = 0;
-    float2 na[D][kA / 2];  // negated anchor coordinates, packed (a_{2m}, a_{2m+1})
-    int aidx[kA];          // anchor index, or kNoAnchor if outside [rb, re)
+    float2 na[D][C::KA / 2];  // negated anchor coordinates, packed (a_{2m}, a_{2m+1})
     for (long long it = beg; it < end; ++it) {
       const int s = (int)((it - beg) & 1);
       int nI = I, nJ = J + 1;
-      if (nJ == g.Mc) { nI = I + 1; nJ = nI * kRatio; }
-      if (tid == 0 && it + 1 < end) issue_chunk<Op, D>(soa, g, nJ, bufs + (s ^ 1) * D * kTP, s ? bar0 : bar1);
+      if (nJ == g.Mc) { nI = I + 1; nJ = nI * C::RATIO; }
+      if (tid == 0 && it + 1 < end) issue_chunk<D, C::TP>(soa, g, nJ, bufs + (s ^ 1) * D * C::TP, s ? bar0 : bar1);
       if (I != curI) {
         curI = I;
 #pragma unroll
-        for (int k = 0; k < kA; ++k) {
-          const int a = I * kTA + k * kThreads + tid;
-          aidx[k] = (a >= g.rb && a < g.re) ? a : kNoAnchor;
+        for (int k = 0; k < C::KA; ++k) {
+          const int a = I * C::TA + k * kThreads + tid;
 #pragma unroll
           for (int c = 0; c < D; ++c) {
             const float v = -__ldg(soa + (long long)c * g.n_pad + a);
@@ -357,12 +466,18 @@ __global__ void __launch_bounds__(kThreads, 2) pair_kernel(const float* __restri
       }
       mbar_wait(s ? bar1 : bar0, (phase >> s) & 1u);
       phase ^= 1u << s;
-      const float* B = bufs + s * D * kTP;
-      const int p0 = J * kTP;
-      const int cnt = min(kTP, g.n - p0);
-      const bool fast = (I * kTA >= g.rb) && ((I + 1) * kTA <= g.re) && (p0 >= (I + 1) * kTA) && (cnt == kTP);
-      if (fast) run_chunk<Op, D, false>(op, B, na, aidx, p0, cnt, g.n);
-      else run_chunk<Op, D, true>(op, B, na, aidx, p0, cnt, g.n);
+      const float* B = bufs + s * D * C::TP;
+      const int p0 = J * C::TP;
+      const int cnt = min(C::TP, g.n - p0);
+      const bool fast =
+          (I * C::TA >= g.rb) && ((I + 1) * C::TA <= g.re) && (p0 >= (I + 1) * C::TA) && (cnt == C::TP);
+      if (clamp) {
+        if (fast) run_chunk<Op, D, C, false, true>(op, B, na, g, I, p0, cnt);
+        else run_chunk<Op, D, C, true, true>(op, B, na, g, I, p0, cnt);
+      } else {
+        if (fast) run_chunk<Op, D, C, false, false>(op, B, na, g, I, p0, cnt);
+        else run_chunk<Op, D, C, true, false>(op, B, na, g, I, p0, cnt);
+      }
       __syncthreads();
       op.after_item(smem, since);
       I = nI;
