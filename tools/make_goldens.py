@@ -23,6 +23,8 @@ GOLDENS = {
     "sdh_uniform_n1048576_nb256_seed2": dict(op="sdh", kind="uniform", n=1 << 20, seed=2, nb=256),
     # 2PCF on the clustered generator at N=1M (r = 0.03), a C3-recipe case small enough for the oracle
     "pcf_clustered_n1048576_r0.03_seed3": dict(op="pcf", kind="clustered", n=1 << 20, seed=3, r=0.03),
+    # BASELINE.json configs[3] recipe at full size: SDH N=2M uniform, 16384 buckets (seed 4)
+    "sdh_uniform_n2097152_nb16384_seed4": dict(op="sdh", kind="uniform", n=1 << 21, seed=4, nb=16384),
     # BASELINE.json configs[0]: SDH N=4096 uniform, 64 buckets (seed 1)
     "sdh_uniform_n4096_nb64_seed1": dict(op="sdh", kind="uniform", n=4096, seed=1, nb=64),
 }
