@@ -1,0 +1,168 @@
+"""GPU parity at BASELINE.json's full sizes, in the launch configuration bench.py times
+(the default tbs.sdh / tbs.pcf / tbs.pairmatrix paths).
+
+Where the O(N^2) oracle is too slow, the check is either (a) against a committed
+golden written by tools/make_goldens.py (oracle only), (b) against the oracle on
+sampled anchor strips (the row-range API computes exactly those pairs), or (c)
+against the O(L^3) exact lattice closed form (oracle.lattice_closed), plus the
+histogram-mass invariant.
+"""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import tbs_inputs as g
+from parity import check_matrix, check_pcf_float, check_sdh_float
+
+pytestmark = pytest.mark.gpu
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def dev(p):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(p)).cuda()
+
+
+def host(t):
+    import torch
+    torch.cuda.synchronize()
+    return t.cpu().numpy()
+
+
+def strips(n, width=48):
+    return [(0, width), (n // 2, n // 2 + width), (n - width, n)]
+
+
+def w_of(nb):
+    return float(np.float32(math.sqrt(3) / nb))
+
+
+# ---------------------------------------------------------------- configs[1]: SDH N=1M, 256 buckets
+def test_sdh_1m_uniform_vs_golden(tbs):
+    gold = json.load(open(os.path.join(GOLD, "sdh_uniform_n1048576_nb256_seed2.json")))
+    p = g.uniform(1 << 20, 2)
+    h = host(tbs.sdh(dev(p), gold["w"], 256)).astype(np.uint64)
+    d = check_sdh_float(h, gold["hist"], gold["amb"])
+    assert int(h.sum()) == (1 << 20) * ((1 << 20) - 1) // 2
+    print("1M golden:", d)
+
+
+def test_sdh_1m_lattice_exact(tbs):
+    """L=100 lattice (N=10^6), w=1, 256 buckets (172 populated): exact vs closed form."""
+    p = g.lattice(100, 2)
+    h = host(tbs.sdh(dev(p), 1.0, 256, lattice=True))
+    assert h.tolist() == oracle.lattice_closed(100, 1, 0, 256)[0].tolist()
+
+
+# ---------------------------------------------------------------- 2PCF (configs[2])
+def test_pcf_1m_clustered_vs_golden(tbs):
+    gold = json.load(open(os.path.join(GOLD, "pcf_clustered_n1048576_r0.03_seed3.json")))
+    p = g.clustered(1 << 20, 3)
+    c = int(host(tbs.pcf(dev(p), 0.03))[0])
+    check_pcf_float(c, gold["count"], gold["amb"])
+
+
+def test_pcf_4m_clustered_strips(tbs):
+    n = 1 << 22
+    p = g.clustered(n, 3)
+    d = dev(p)
+    for rows in strips(n):
+        c = int(host(tbs.pcf(d, 0.03, rows=rows))[0])
+        co, amb = oracle.pcf(p, 0.03, rows=rows)
+        check_pcf_float(c, co, amb)
+    total = int(host(tbs.pcf(d, 0.03))[0])
+    assert total > 2 ** 32            # the count needs the u64 path
+    acc = 0
+    for r in range(8):                 # the 8-rank partition sums to the single-GPU count exactly
+        acc += int(host(tbs.pcf(d, 0.03, rows=tbs.rank_rows(n, 8, r)))[0])
+    assert acc == total
+
+
+def test_pcf_4m_lattice_exact(tbs):
+    """L=160 lattice (N=4,096,000), r=10 (r^2 = 100 exact): exact vs closed form."""
+    p = g.lattice(160, 6)
+    c = int(host(tbs.pcf(dev(p), 10.0))[0])
+    assert c == oracle.lattice_closed(160, 1, 0, 1, r2=100)[1]
+
+
+# ---------------------------------------------------------------- configs[3]: N=2M, 16384 buckets
+@pytest.mark.parametrize("mode", [None, "global"])
+def test_sdh_2m_16k_lattice_exact(tbs, mode):
+    """L=128 lattice (N=2^21), w=2^-6, 16384 buckets (highest bucket 14078): exact vs closed form,
+    default (smem) output stage and the partially privatised global histogram."""
+    p = g.lattice(128, 4)
+    h = host(tbs.sdh(dev(p), 2.0 ** -6, 16384, lattice=True, hist_mode=mode))
+    ref = oracle.lattice_closed(128, 1, 6, 16384)[0]
+    assert h.tolist() == ref.tolist()
+    assert int(np.nonzero(ref)[0].max()) == 14078      # floor(64 * sqrt(3) * 127)
+
+
+@pytest.mark.parametrize("mode", [None, "global"])
+def test_sdh_2m_16k_uniform(tbs, mode):
+    n, nb = 1 << 21, 16384
+    p = g.uniform(n, 4)
+    d = dev(p)
+    h = host(tbs.sdh(d, w_of(nb), nb, hist_mode=mode)).astype(np.uint64)
+    assert int(h.sum()) == n * (n - 1) // 2
+    gp = os.path.join(GOLD, "sdh_uniform_n2097152_nb16384_seed4.json")
+    if os.path.exists(gp):
+        gold = json.load(open(gp))
+        check_sdh_float(h, gold["hist"], gold["amb"])
+    for rows in strips(n, 32):
+        hs = host(tbs.sdh(d, w_of(nb), nb, rows=rows, hist_mode=mode))
+        ho, amb = oracle.sdh(p, w_of(nb), nb, rows=rows)
+        check_sdh_float(hs, ho, amb)
+
+
+# ---------------------------------------------------------------- north-star line: SDH N=4M, 256 buckets
+def test_sdh_4m_uniform_strips_and_mass(tbs):
+    n = 1 << 22
+    p = g.uniform(n, 6)
+    d = dev(p)
+    h = host(tbs.sdh(d, w_of(256), 256))
+    assert int(h.sum()) == n * (n - 1) // 2
+    for rows in strips(n):
+        hs = host(tbs.sdh(d, w_of(256), 256, rows=rows))
+        ho, amb = oracle.sdh(p, w_of(256), 256, rows=rows)
+        check_sdh_float(hs, ho, amb)
+
+
+def test_sdh_4m_lattice_exact(tbs):
+    """L=160 lattice (N=4,096,000), w=1, 256 buckets: d_max = 275.4 so buckets >= 256 clamp
+    into 255 (the clamp path); exact vs closed form."""
+    p = g.lattice(160, 6)
+    h = host(tbs.sdh(dev(p), 1.0, 256, lattice=True))
+    assert h.tolist() == oracle.lattice_closed(160, 1, 0, 256)[0].tolist()
+
+
+def test_sdh_4m_clustered_float_mass_strips(tbs):
+    n = 1 << 22
+    p = g.clustered(n, 3)
+    d = dev(p)
+    h = host(tbs.sdh(d, w_of(256), 256))
+    assert int(h.sum()) == n * (n - 1) // 2
+    rows = (n // 3, n // 3 + 48)
+    hs = host(tbs.sdh(d, w_of(256), 256, rows=rows))
+    ho, amb = oracle.sdh(p, w_of(256), 256, rows=rows)
+    check_sdh_float(hs, ho, amb)
+
+
+# ---------------------------------------------------------------- configs[4]: Type-III N=64K
+def test_pairmatrix_64k_sampled_rows(tbs):
+    import torch
+    n = 1 << 16
+    p = g.uniform(n, 5)
+    out = tbs.pairmatrix(dev(p), 1.0)                      # 17.2 GB fp32 on the device
+    rng = np.random.default_rng(0)
+    rows = sorted(set([0, 1, n - 1] + rng.integers(0, n, 253).tolist()))
+    idx = torch.tensor(rows, device=out.device)
+    got = host(out.index_select(0, idx))
+    del out
+    torch.cuda.empty_cache()
+    for k, r in enumerate(rows):
+        ref = oracle.pairmatrix(p, 1.0, rows=(r, r + 1))[0]
+        check_matrix(got[k], ref)
