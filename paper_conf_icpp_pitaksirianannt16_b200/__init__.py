@@ -109,6 +109,25 @@ def rank_rows(n: int, world: int, rank: int) -> tuple[int, int]:
     return b.value, e.value
 
 
+# ---------------------------------------------------------------- multi-GPU combine
+def partition(n: int, group=None, rows=None):
+    """Anchor rows this rank owns: the pair-balanced strip of `group`, else `rows`."""
+    if group is None:
+        return rows
+    import torch.distributed as dist
+    return rank_rows(n, dist.get_world_size(group), dist.get_rank(group))
+
+
+def combine(partial, group=None):
+    """The method's one exchange step: sum the per-rank int64 partial
+    histograms / counts with a single all_reduce (NCCL over NVLink on GPUs). Integer
+    sums are order-independent, so the result is bit-identical to one GPU."""
+    if group is not None:
+        import torch.distributed as dist
+        dist.all_reduce(partial, op=dist.ReduceOp.SUM, group=group)
+    return partial
+
+
 # ---------------------------------------------------------------- device (torch) API
 def _torch():
     import torch
@@ -143,31 +162,19 @@ def sdh(points, bucket_width: float, nbuckets: int, *, rows=None, lattice: bool 
     """
     torch = _torch()
     flags = (TBS_EXACT_LATTICE if lattice else 0) | HIST_MODES[hist_mode] | (TBS_FORCE_CLAMP if force_clamp else 0)
-    if group is not None:
-        import torch.distributed as dist
-        rows = rank_rows(points.shape[0], dist.get_world_size(group), dist.get_rank(group))
-    a, _ = _args(points, rows, flags, stream, events)
+    a, _ = _args(points, partition(points.shape[0], group, rows), flags, stream, events)
     h = out if out is not None else torch.empty(nbuckets, dtype=torch.int64, device=points.device)
     _check(lib().tbs_sdh_ex(ctypes.byref(a), float(bucket_width), int(nbuckets), h.data_ptr()), "tbs_sdh_ex")
-    if group is not None:
-        import torch.distributed as dist
-        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
-    return h
+    return combine(h, group)
 
 
 def pcf(points, radius: float, *, rows=None, out=None, stream=None, events=None, group=None):
     """2-point correlation count (Type-I): #{i<j : d < radius}, int64[1] on points.device."""
     torch = _torch()
-    if group is not None:
-        import torch.distributed as dist
-        rows = rank_rows(points.shape[0], dist.get_world_size(group), dist.get_rank(group))
-    a, _ = _args(points, rows, 0, stream, events)
+    a, _ = _args(points, partition(points.shape[0], group, rows), 0, stream, events)
     c = out if out is not None else torch.empty(1, dtype=torch.int64, device=points.device)
     _check(lib().tbs_pcf_ex(ctypes.byref(a), float(radius), c.data_ptr()), "tbs_pcf_ex")
-    if group is not None:
-        import torch.distributed as dist
-        dist.all_reduce(c, op=dist.ReduceOp.SUM, group=group)
-    return c
+    return combine(c, group)
 
 
 def pairmatrix(points, gamma: float = 1.0, *, kernel: str = "gaussian", rows=None, out=None, stream=None,
