@@ -49,7 +49,8 @@ METRIC = "SDH pair-distances/sec (G pairs/s) at N=1M–4M, 1/2/4/8 B200, % of ro
 # Roofline denominators: B200 unit counts x max SM clock.
 SMS = 148
 FP32_LANES_PER_CLK_SM = 128        # FFMA/FADD lanes per SM per clock (FFMA2 issues half as often, same lanes)
-ATOMS_LANES_PER_CLK_SM = 16        # shared-memory atomic lanes per SM per clock (measured 14.8, tools/peaks.cu)
+ATOMS_LANES_PER_CLK_SM = 32        # conflict-free shared atomics: 1 warp-instr/clk/SM (31.5 measured, tools/peaks.cu)
+MUFU_LANES_PER_CLK_SM = 16         # XU pipe (sqrt/rsqrt/ex2): 15.9 measured; one sqrt per SDH pair
 
 
 def peaks():
@@ -63,6 +64,7 @@ def peaks():
         f_max=f_max,
         fp32=SMS * FP32_LANES_PER_CLK_SM * f_max,
         atoms=SMS * ATOMS_LANES_PER_CLK_SM * f_max,
+        mufu=SMS * MUFU_LANES_PER_CLK_SM * f_max,
         hbm=float(mp.get("hbm_gbs", 6650.0)) * 1e9,
         hbm_src="MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in mp else "fallback 6.65 TB/s (B200_PROFILING.md)",
     )
@@ -295,6 +297,9 @@ def main():
                 "frac": pairs_s / peak, "peak_source": f"{bound_note}; 148 SMs x unit lanes/clk x "
                                                       f"{pk['f_max'] / 1e6:.0f} MHz (DESIGN.md §Roofline)",
                 "frac_fp32": pairs_s * 6 / pk["fp32"]}
+        if op != "pcf":
+            roof["mufu_cap"] = pk["mufu"] / 1e9         # one MUFU.SQRT per pair: this design's ceiling
+            roof["frac_of_mufu_cap"] = pairs_s / pk["mufu"]
     roof["traffic"] = None
     prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(prof):

@@ -8,6 +8,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <type_traits>
@@ -130,6 +131,11 @@ int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op
   int occ = 0;
   TBS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, (size_t)smem));
   if (occ < 1) return fail(TBS_EUNSUPPORTED, "pair kernel cannot be resident (smem %lld)", smem);
+  static const int occ_cap = [] {  // experiments only: TBS_OCC caps resident CTAs per SM
+    const char* e = getenv("TBS_OCC");
+    return e ? atoi(e) : 0;
+  }();
+  if (occ_cap > 0 && occ_cap < occ) occ = occ_cap;
   long long grid = (long long)dev.sms * occ;
   if (grid > g.items) grid = g.items;
   if (eb) TBS_CUDA(cudaEventRecord(eb, st));

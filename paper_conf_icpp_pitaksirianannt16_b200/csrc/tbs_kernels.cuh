@@ -25,9 +25,6 @@ namespace tbs {
 #ifndef TBS_PUNROLL
 #define TBS_PUNROLL 1                      // partner-quad loop unroll (software-pipelining freedom)
 #endif
-#ifndef TBS_ADDR_MODE
-#define TBS_ADDR_MODE 0                    // 0: LEA from the floor's bits; 1: FADD2 into a binade + IADD
-#endif
 constexpr int kThreads = 256;              // 8 warps per CTA
 constexpr int kPUnroll = TBS_PUNROLL;
 constexpr int kWarps = kThreads / 32;
@@ -221,17 +218,15 @@ struct SdhSmemOp {
         y.x = fminf(y.x, ymax);
         y.y = fminf(y.y, ymax);
       }
-#if TBS_ADDR_MODE == 1
-      const float2 z = __fadd2_rn(y, make_float2(zc, zc));
-      // uniform part recomputed from the smem symbol so ptxas may fold it into [R + UR]
-      const uint32_t ub = smem_addr(tbs_smem) - __float_as_uint((float)(1 << E));
-      ad0 = __float_as_uint(z.x) + ub;
-      ad1 = __float_as_uint(z.y) + ub;
-#else
-      // bits(y) = 2^23's bits + k: one shift-add (LEA) gives base + 4 (k R + lane_r)
-      ad0 = (__float_as_uint(y.x) << (LOG2R + 2)) + base;
-      ad1 = (__float_as_uint(y.y) << (LOG2R + 2)) + base;
-#endif
+      // bits(y) = bits(2^23) + k. Funnel shift (bits << S) | (lo >> (32-S)) with S = log2(4R)
+      // and lo = 4 lane_r << (32-S) gives 4 (k R + lane_r) + (bits(2^23) << S); the
+      // CTA-uniform correction (smem base - (bits(2^23) << S)) is recomputed from the smem
+      // symbol so ptxas fuses shift + add into one ALU LEA.HI with a uniform operand.
+      constexpr int S = LOG2R + 2;
+      const uint32_t lo = (uint32_t)((threadIdx.x & (R - 1)) * 4) << (32 - S);
+      const uint32_t ub = smem_addr(tbs_smem) - (kMagic << S);
+      ad0 = __funnelshift_l(lo, __float_as_uint(y.x), S) + ub;
+      ad1 = __funnelshift_l(lo, __float_as_uint(y.y), S) + ub;
     } else {
       const uint32_t b0 = min(bucket_bits(s.x), bmax), b1 = min(bucket_bits(s.y), bmax);
       ad0 = (b0 << (LOG2R + 2)) + base;

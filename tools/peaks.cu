@@ -122,6 +122,24 @@ __global__ void k_atoms(unsigned* out) {
   if (threadIdx.x == 0 && h[5] == 0xffffffffu) out[0] = h[0];
 }
 
+// Pure shared atomics: 8 fixed lane-private addresses per thread, no ALU per atomic.
+__global__ void k_atoms_pure(unsigned* out) {
+  extern __shared__ unsigned h[];
+  const int lane = threadIdx.x & 31;
+  for (int i = threadIdx.x; i < 64 * 32; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  uint32_t a[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c)
+    a[c] = (uint32_t)__cvta_generic_to_shared(h + ((threadIdx.x * 7 + c * 13) & 63) * 32 + lane);
+  for (int i = 0; i < ITERS / 4; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(a[c]));
+  }
+  __syncthreads();
+  if (threadIdx.x == 0 && h[5] == 0xffffffffu) out[0] = h[0];
+}
+
 // ---- LDS.128 broadcast ---------------------------------------------------------
 __global__ void k_lds128(float* out) {
   __shared__ float4 s[1024];
@@ -174,6 +192,7 @@ int main() {
   rep("mufu_ex2", it, timeit([&] { k_mufu<2><<<blocks, threads>>>(dout); }));
   double at = (double)(ITERS / 4) * 8 * thr;
   rep("atoms_lane_private", at, timeit([&] { k_atoms<0><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("atoms_pure_lane_private", at, timeit([&] { k_atoms_pure<<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
   rep("atoms_random_256", at, timeit([&] { k_atoms<1><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
   rep("atoms_same_addr", at, timeit([&] { k_atoms<2><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
   rep("lds128_bcast_instr", (double)ITERS * thr, timeit([&] { k_lds128<<<blocks, threads>>>(dout); }));

@@ -14,10 +14,10 @@ for f in re.split(r'\n\s+Function : ', txt):
     lines = [l for l in f.split('\n') if re.search(r'/\*[0-9a-f]{4}\*/', l)]
     addr = lambda x: int(re.search(r'/\*([0-9a-f]{4,})\*/', x).group(1), 16)
     for l in lines:
-        m = re.search(r'/\*([0-9a-f]{4,})\*/\s+(@!?U?P\w+\s+)?BRA(\.\S+)?\s+(?:`?\(?)?0x([0-9a-f]+)', l)
+        m = re.search(r'/\*([0-9a-f]{4,})\*/\s+(@!?U?P\w+\s+)?BRA(\.\S+)?\s+(?:!?U?P\w+,\s*)?(?:`?\(?)?0x([0-9a-f]+)', l)
         if m:
             src, dst = int(m.group(1), 16), int(m.group(4), 16)
-            if dst < src and src - dst > 0x400:
+            if dst < src and src - dst > 0x300:
                 body = [x for x in lines if dst <= addr(x) <= src]
                 ops = {}
                 for x in body:
