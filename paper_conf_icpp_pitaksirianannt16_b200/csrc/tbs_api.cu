@@ -53,6 +53,12 @@ using namespace tbs;
 using SdhCfg = Cfg<TBS_SDH_CFG>;
 using PcfCfg = Cfg<TBS_PCF_CFG>;
 using LatCfg = Cfg<TBS_LAT_CFG>;
+// Small problems (fewer work items than ~2 per SM with the main configs): finer tiles so
+// the grid covers the GPU (BASELINE configs[0], N = 4096, is launch/latency-bound).
+#ifndef TBS_SMALL_TP
+#define TBS_SMALL_TP 128
+#endif
+using SmallCfg = Cfg<2, TBS_SMALL_TP, 4>;
 
 namespace {
 
@@ -127,9 +133,17 @@ int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op
   const Geom g = make_geom(a->n, a->row_begin, a->row_end, C::TA, C::TP);
   const long long smem = ((op.smem_bytes() + 127) & ~127ll) + 2ll * D * C::TP * 4 + 16;
   if (smem > dev.smem_optin) return fail(TBS_EUNSUPPORTED, "pair kernel needs %lld B smem > %d", smem, dev.smem_optin);
-  TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  // per-instantiation cache of the attribute + occupancy query (host overhead of small calls)
+  struct OccCache { int dev = -1; long long smem = -1; int occ = 0; };
+  static thread_local OccCache cache;
   int occ = 0;
-  TBS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, (size_t)smem));
+  if (cache.dev == dev.id && cache.smem == smem) {
+    occ = cache.occ;
+  } else {
+    TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    TBS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, (size_t)smem));
+    cache = OccCache{dev.id, smem, occ};
+  }
   if (occ < 1) return fail(TBS_EUNSUPPORTED, "pair kernel cannot be resident (smem %lld)", smem);
   static const int occ_cap = [] {  // experiments only: TBS_OCC caps resident CTAs per SM
     const char* e = getenv("TBS_OCC");
@@ -213,8 +227,7 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
     g_launches.fetch_add(1);
     return TBS_OK;
   }
-  using C = typename std::conditional<LAT, LatCfg, SdhCfg>::type;
-  auto fill = [&](auto& op, int R) {
+  auto fill = [&](auto& op, int R, long long ka_tp) {
     op.nb = nb;
     op.rows = LAT ? nb : nb + kGuard;
     op.inv_w = (float)(1.0 / (double)w);
@@ -223,13 +236,31 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
     op.sh = 2 * j;
     op.hist = hist;
     // per item, a replica receives at most (32/R) lanes x kWarps x KA x TP increments
-    const long long per_item = (long long)(32 / R) * kWarps * C::KA * C::TP;
+    const long long per_item = (long long)(32 / R) * kWarps * ka_tp;
     op.flush_every = (int)std::max<long long>(1, (0xffffffffll / per_item) - 1);
   };
+  using C = typename std::conditional<LAT, LatCfg, SdhCfg>::type;
+  const bool small = !LAT && make_geom(g->n, g->row_begin, g->row_end, C::TA, C::TP).items < 2ll * dev.sms;
   switch (pl.log2r) {
-    case 5: { SdhSmemOp<5, LAT> op{}; fill(op, 32); return launch_pair<SdhSmemOp<5, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee); }
-    case 2: { SdhSmemOp<2, LAT> op{}; fill(op, 4); return launch_pair<SdhSmemOp<2, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee); }
-    default: { SdhSmemOp<0, LAT> op{}; fill(op, 1); return launch_pair<SdhSmemOp<0, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee); }
+    case 5: {
+      SdhSmemOp<5, LAT> op{};
+      if (small) {
+        fill(op, 32, (long long)SmallCfg::KA * SmallCfg::TP);
+        return launch_pair<SdhSmemOp<5, LAT>, D, SmallCfg>(dev, soa, g, op, bbox, st, eb, ee);
+      }
+      fill(op, 32, (long long)C::KA * C::TP);
+      return launch_pair<SdhSmemOp<5, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+    }
+    case 2: {
+      SdhSmemOp<2, LAT> op{};
+      fill(op, 4, (long long)C::KA * C::TP);
+      return launch_pair<SdhSmemOp<2, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+    }
+    default: {
+      SdhSmemOp<0, LAT> op{};
+      fill(op, 1, (long long)C::KA * C::TP);
+      return launch_pair<SdhSmemOp<0, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+    }
   }
 }
 
@@ -323,8 +354,13 @@ int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
     op.r2 = (float)((double)r * (double)r);
     op.count = c;
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
-    rc = D == 3 ? launch_pair<PcfOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee)
-                 : launch_pair<PcfOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee);
+    const bool small = make_geom(a->n, a->row_begin, a->row_end, PcfCfg::TA, PcfCfg::TP).items < 2ll * dev.sms;
+    if (small)
+      rc = D == 3 ? launch_pair<PcfOp, 3, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee)
+                  : launch_pair<PcfOp, 4, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee);
+    else
+      rc = D == 3 ? launch_pair<PcfOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee)
+                  : launch_pair<PcfOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee);
   }
   if (soa) cudaFreeAsync(soa, st);
   return rc;

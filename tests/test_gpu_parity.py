@@ -48,6 +48,18 @@ def test_sdh_uniform_ragged(tbs, n):
     check_sdh_float(h, ho, amb)
 
 
+@pytest.mark.parametrize("n", [20001, 30000])
+def test_sdh_main_config_ragged(tbs, n):
+    """Sizes above the small-problem switch: the main tile configuration, ragged tail."""
+    p = g.clustered(n, 31)
+    h = sdh_gpu(tbs, p, w_of(256), 256)
+    ho, amb = oracle.sdh(p, w_of(256), 256)
+    check_sdh_float(h, ho, amb)
+    c = int(tbs.pcf(dev(p), 0.02).item())
+    co, ca = oracle.pcf(p, 0.02)
+    check_pcf_float(c, co, ca)
+
+
 def test_sdh_config1(tbs):
     """BASELINE.json configs[0]: N=4096 uniform, 64 buckets (golden from tools/make_goldens.py)."""
     import json, os
