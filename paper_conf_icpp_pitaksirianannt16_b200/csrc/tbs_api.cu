@@ -56,7 +56,7 @@ using LatCfg = Cfg<TBS_LAT_CFG>;
 // Small problems (fewer work items than ~2 per SM with the main configs): finer tiles so
 // the grid covers the GPU (BASELINE configs[0], N = 4096, is launch/latency-bound).
 #ifndef TBS_SMALL_TP
-#define TBS_SMALL_TP 128
+#define TBS_SMALL_TP 64
 #endif
 using SmallCfg = Cfg<2, TBS_SMALL_TP, 4>;
 

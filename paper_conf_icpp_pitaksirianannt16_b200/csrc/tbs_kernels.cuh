@@ -189,23 +189,41 @@ struct SdhSmemOp {
     ymax = kMagicF + (float)(nb - 1);
   }
   __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
+  // Float mode: true if the clamp to nb-1 is needed. Lattice mode: true if the general
+  // (u64) exact fix-up is needed; false when the bounding box proves every product of
+  // the fix-up fits 32 bits (s < 2^23, 4^j s < 2^32, ((nb+1) m)^2 < 2^32).
   __device__ __forceinline__ bool needs_clamp(const uint32_t* bbox, int D) const {
-    if (LATTICE) return true;
+    if (LATTICE) {
+      const float dmax = bbox_diameter(bbox, D);
+      const double smax = (double)dmax * (double)dmax;
+      const double em = (double)(nb + 1) * (double)m;
+      return !(smax < 8388608.0 && smax * (double)(1ull << sh) < 4294967296.0 && em * em < 4294967296.0);
+    }
     const float dmax = bbox_diameter(bbox, D);
     return !(dmax * inv_w < (float)(nb + kGuard - 2));
   }
 
-  __device__ __forceinline__ uint32_t bucket_bits(float s) const {
-    // lattice: s is an exact integer < 2^24. fp32 estimate, then exact integer fix-up by one step.
-    uint32_t si = __float2uint_rz(s);
-    float q = sqrt_approx(s);
+  // Lattice bucket: s is an exact integer (< 2^24; < 2^23 on the 32-bit path). fp32
+  // estimate k0 = floor(sqrt(s) 2^j / m), then one exact integer step each way against
+  // (k m)^2 <= 4^j s. Returns the clamped bucket index.
+  template <bool GENERAL>
+  __device__ __forceinline__ uint32_t lattice_bucket(float s) const {
+    const float q = sqrt_approx(s);
     int k = min((int)(__float_as_uint(__fmaf_rd(q, scale, kMagicF)) - kMagic), nb);
-    unsigned long long S = (unsigned long long)si << sh;
-    unsigned long long e1 = (unsigned long long)(k + 1) * (unsigned long long)m;
-    k += (e1 * e1 <= S) ? 1 : 0;
-    unsigned long long e0 = (unsigned long long)k * (unsigned long long)m;
-    k -= (e0 * e0 > S) ? 1 : 0;
-    return kMagic + (uint32_t)k;
+    if (GENERAL) {
+      const unsigned long long S = (unsigned long long)__float2uint_rz(s) << sh;
+      const unsigned long long e1 = (unsigned long long)(k + 1) * (unsigned long long)m;
+      k += (e1 * e1 <= S) ? 1 : 0;
+      const unsigned long long e0 = (unsigned long long)k * (unsigned long long)m;
+      k -= (e0 * e0 > S) ? 1 : 0;
+    } else {
+      const uint32_t S = (__float_as_uint(__fadd_rn(s, kMagicF)) - kMagic) << sh;   // exact for s < 2^23
+      const uint32_t e1 = (uint32_t)(k + 1) * (uint32_t)m;
+      k += (e1 * e1 <= S) ? 1 : 0;
+      const uint32_t e0 = (uint32_t)k * (uint32_t)m;
+      k -= (e0 * e0 > S) ? 1 : 0;
+    }
+    return (uint32_t)min(k, nb - 1);
   }
 
   template <bool MASKED, bool CLAMP>
@@ -228,9 +246,10 @@ struct SdhSmemOp {
       ad0 = __funnelshift_l(lo, __float_as_uint(y.x), S) + ub;
       ad1 = __funnelshift_l(lo, __float_as_uint(y.y), S) + ub;
     } else {
-      const uint32_t b0 = min(bucket_bits(s.x), bmax), b1 = min(bucket_bits(s.y), bmax);
-      ad0 = (b0 << (LOG2R + 2)) + base;
-      ad1 = (b1 << (LOG2R + 2)) + base;
+      const uint32_t k0 = lattice_bucket<CLAMP>(s.x), k1 = lattice_bucket<CLAMP>(s.y);
+      const uint32_t lb = smem_addr(tbs_smem) + (uint32_t)((threadIdx.x & (R - 1)) * 4);
+      ad0 = (k0 << (LOG2R + 2)) + lb;
+      ad1 = (k1 << (LOG2R + 2)) + lb;
     }
     if (MASKED) {
       red_smem_inc_gt(ad0, pv, a0);
