@@ -232,6 +232,7 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
     op.rows = LAT ? nb : nb + kGuard;
     op.inv_w = (float)(1.0 / (double)w);
     op.scale = (float)std::ldexp(1.0 / (double)m, j);
+    op.mj = (float)std::ldexp((double)m, -j);
     op.m = (int)m;
     op.sh = 2 * j;
     op.hist = hist;

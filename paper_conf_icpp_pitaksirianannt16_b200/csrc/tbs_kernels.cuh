@@ -189,28 +189,35 @@ struct SdhSmemOp {
     ymax = kMagicF + (float)(nb - 1);
   }
   __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
-  // Float mode: true if the clamp to nb-1 is needed. Lattice mode: true if the general
-  // (u64) exact fix-up is needed; false when the bounding box proves every product of
-  // the fix-up fits 32 bits (s < 2^23, 4^j s < 2^32, ((nb+1) m)^2 < 2^32).
-  __device__ __forceinline__ bool needs_clamp(const uint32_t* bbox, int D) const {
-    if (LATTICE) {
-      const float dmax = bbox_diameter(bbox, D);
-      const double smax = (double)dmax * (double)dmax;
-      const double em = (double)(nb + 1) * (double)m;
-      return !(smax < 8388608.0 && smax * (double)(1ull << sh) < 4294967296.0 && em * em < 4294967296.0);
-    }
+  // Kernel-uniform code variant, chosen once from the loader's bounding box:
+  //   float mode:   0 = no clamp (every k < nb + kGuard is proven), 1 = clamp to nb-1;
+  //   lattice mode: exact fix-up in 0 = fp32 (all products < 2^24, exact in float),
+  //                 1 = 32-bit integers, 2 = 64-bit integers (general).
+  static constexpr int kVariants = LATTICE ? 3 : 2;
+  float mj;           // lattice: m * 2^-j (exact)
+  __device__ __forceinline__ int variant(const uint32_t* bbox, int D) const {
     const float dmax = bbox_diameter(bbox, D);
-    return !(dmax * inv_w < (float)(nb + kGuard - 2));
+    if (LATTICE) {
+      const double smax = (double)dmax * (double)dmax;             // >= every s (integer data)
+      const double S = smax * (double)(1ull << sh);                // 4^j s_max
+      const double kmax = floor(sqrt(S) / (double)m) + 2.0;         // estimate + fix-up reach
+      const double e = fmax(kmax, (double)(nb + 1)) * (double)m;
+      if (smax < 8388608.0 && S < 16777216.0 && e * e < 16777216.0) return 0;
+      const double em = (double)(nb + 1) * (double)m;
+      if (smax < 8388608.0 && S < 4294967296.0 && em * em < 4294967296.0) return 1;
+      return 2;
+    }
+    return (dmax * inv_w < (float)(nb + kGuard - 2)) ? 0 : 1;
   }
 
   // Lattice bucket: s is an exact integer (< 2^24; < 2^23 on the 32-bit path). fp32
   // estimate k0 = floor(sqrt(s) 2^j / m), then one exact integer step each way against
   // (k m)^2 <= 4^j s. Returns the clamped bucket index.
-  template <bool GENERAL>
+  template <int V>
   __device__ __forceinline__ uint32_t lattice_bucket(float s) const {
     const float q = sqrt_approx(s);
     int k = min((int)(__float_as_uint(__fmaf_rd(q, scale, kMagicF)) - kMagic), nb);
-    if (GENERAL) {
+    if (V == 2) {
       const unsigned long long S = (unsigned long long)__float2uint_rz(s) << sh;
       const unsigned long long e1 = (unsigned long long)(k + 1) * (unsigned long long)m;
       k += (e1 * e1 <= S) ? 1 : 0;
@@ -226,13 +233,29 @@ struct SdhSmemOp {
     return (uint32_t)min(k, nb - 1);
   }
 
-  template <bool MASKED, bool CLAMP>
+  // Lattice, fp32 fix-up for two pairs: with e = k m 2^-j, e^2 - s = ((k m)^2 - 4^j s) / 4^j
+  // is an integer < 2^24 scaled by a power of two, so one FFMA computes it exactly.
+  __device__ __forceinline__ void lattice_bucket2_f32(float2 s, uint32_t& k0, uint32_t& k1) const {
+    const float2 q = make_float2(sqrt_approx(s.x), sqrt_approx(s.y));
+    const float2 y = __ffma2_rd(q, make_float2(scale, scale), make_float2(kMagicF, kMagicF));
+    const float2 kf = __fadd2_rn(y, make_float2(-kMagicF, -kMagicF));
+    const float2 e0 = __fmul2_rn(kf, make_float2(mj, mj));
+    const float2 e1 = __fadd2_rn(e0, make_float2(mj, mj));
+    const float2 ns = make_float2(-s.x, -s.y);
+    const float2 d1 = __ffma2_rn(e1, e1, ns);
+    const float2 d0 = __ffma2_rn(e0, e0, ns);
+    const int b0 = (int)(__float_as_uint(y.x) - kMagic), b1 = (int)(__float_as_uint(y.y) - kMagic);
+    k0 = (uint32_t)min(b0 + (d1.x <= 0.f ? 1 : 0) - (d0.x > 0.f ? 1 : 0), nb - 1);
+    k1 = (uint32_t)min(b1 + (d1.y <= 0.f ? 1 : 0) - (d0.y > 0.f ? 1 : 0), nb - 1);
+  }
+
+  template <bool MASKED, int V>
   __device__ __forceinline__ void pair2(float2 s, int pv, int a0, int a1) {
     uint32_t ad0, ad1;
     if (!LATTICE) {
       const float2 q = make_float2(sqrt_approx(s.x), sqrt_approx(s.y));
       float2 y = __ffma2_rd(q, make_float2(inv_w, inv_w), make_float2(kMagicF, kMagicF));
-      if (CLAMP) {
+      if (V == 1) {
         y.x = fminf(y.x, ymax);
         y.y = fminf(y.y, ymax);
       }
@@ -246,7 +269,13 @@ struct SdhSmemOp {
       ad0 = __funnelshift_l(lo, __float_as_uint(y.x), S) + ub;
       ad1 = __funnelshift_l(lo, __float_as_uint(y.y), S) + ub;
     } else {
-      const uint32_t k0 = lattice_bucket<CLAMP>(s.x), k1 = lattice_bucket<CLAMP>(s.y);
+      uint32_t k0, k1;
+      if (V == 0) {
+        lattice_bucket2_f32(s, k0, k1);
+      } else {
+        k0 = lattice_bucket<V>(s.x);
+        k1 = lattice_bucket<V>(s.y);
+      }
       const uint32_t lb = smem_addr(tbs_smem) + (uint32_t)((threadIdx.x & (R - 1)) * 4);
       ad0 = (k0 << (LOG2R + 2)) + lb;
       ad1 = (k1 << (LOG2R + 2)) + lb;
@@ -317,8 +346,9 @@ struct SdhGlobalOp {
     }
     return min(k, nb - 1);
   }
-  __device__ __forceinline__ bool needs_clamp(const uint32_t*, int) const { return false; }
-  template <bool MASKED, bool CLAMP>
+  static constexpr int kVariants = 1;
+  __device__ __forceinline__ int variant(const uint32_t*, int) const { return 0; }
+  template <bool MASKED, int V>
   __device__ __forceinline__ void pair2(float2 s, int pv, int a0, int a1) {
     unsigned long long* p0 = mine + bucket(s.x);
     unsigned long long* p1 = mine + bucket(s.y);
@@ -345,8 +375,9 @@ struct PcfOp {
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) { c = 0u; total = 0ull; }
   __device__ __forceinline__ float2 bias() const { return make_float2(-r2, -r2); }
-  __device__ __forceinline__ bool needs_clamp(const uint32_t*, int) const { return false; }
-  template <bool MASKED, bool CLAMP>
+  static constexpr int kVariants = 1;
+  __device__ __forceinline__ int variant(const uint32_t*, int) const { return 0; }
+  template <bool MASKED, int V>
   __device__ __forceinline__ void pair2(float2 t, int pv, int a0, int a1) {
     uint32_t s0 = __float_as_uint(t.x) >> 31, s1 = __float_as_uint(t.y) >> 31;
     if (MASKED) {
@@ -391,7 +422,7 @@ __device__ __forceinline__ void issue_chunk(const float* __restrict__ soa, const
     bulk_g2s(smem_addr(dst + c * TP), soa + (long long)c * g.n_pad + (long long)J * TP, TP * 4, bar);
 }
 
-template <class Op, int D, class C, bool MASKED, bool CLAMP>
+template <class Op, int D, class C, bool MASKED, int V>
 __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, const float2 (&na)[D][C::KA / 2],
                                           const Geom& g, int I, int p0, int cnt) {
   // masked items only: anchor index or kNoAnchor outside [rb, re) (built here so the
@@ -426,7 +457,7 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
           d = __fadd2_rn(na[c][m], make_float2(c4[c][q], c4[c][q]));
           s = __ffma2_rn(d, d, s);
         }
-        op.template pair2<MASKED, CLAMP>(s, pv, MASKED ? aidx[2 * m] : 0, MASKED ? aidx[2 * m + 1] : 0);
+        op.template pair2<MASKED, V>(s, pv, MASKED ? aidx[2 * m] : 0, MASKED ? aidx[2 * m + 1] : 0);
       }
     }
   }
@@ -443,7 +474,7 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
   const int tid = threadIdx.x;
 
   op.init(smem);
-  const bool clamp = op.needs_clamp(bbox, D);
+  const int variant = op.variant(bbox, D);
   if (tid == 0) {
     mbar_init(bar0, 1);
     mbar_init(bar1, 1);
@@ -485,13 +516,24 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
       const int cnt = min(C::TP, g.n - p0);
       const bool fast =
           (I * C::TA >= g.rb) && ((I + 1) * C::TA <= g.re) && (p0 >= (I + 1) * C::TA) && (cnt == C::TP);
-      if (clamp) {
-        if (fast) run_chunk<Op, D, C, false, true>(op, B, na, g, I, p0, cnt);
-        else run_chunk<Op, D, C, true, true>(op, B, na, g, I, p0, cnt);
-      } else {
-        if (fast) run_chunk<Op, D, C, false, false>(op, B, na, g, I, p0, cnt);
-        else run_chunk<Op, D, C, true, false>(op, B, na, g, I, p0, cnt);
+      if constexpr (Op::kVariants > 2) {
+        if (variant == 2) {
+          if (fast) run_chunk<Op, D, C, false, 2>(op, B, na, g, I, p0, cnt);
+          else run_chunk<Op, D, C, true, 2>(op, B, na, g, I, p0, cnt);
+          goto item_done;
+        }
       }
+      if constexpr (Op::kVariants > 1) {
+        if (variant == 1) {
+          if (fast) run_chunk<Op, D, C, false, 1>(op, B, na, g, I, p0, cnt);
+          else run_chunk<Op, D, C, true, 1>(op, B, na, g, I, p0, cnt);
+          goto item_done;
+        }
+      }
+      if (fast) run_chunk<Op, D, C, false, 0>(op, B, na, g, I, p0, cnt);
+      else run_chunk<Op, D, C, true, 0>(op, B, na, g, I, p0, cnt);
+      goto item_done;  // (keeps the label referenced for single-variant ops)
+    item_done:
       __syncthreads();
       op.after_item(smem, since);
       I = nI;
