@@ -12,6 +12,7 @@
 #include <cstring>
 #include <string>
 #include <type_traits>
+#include <vector>
 
 #include "tbs.h"
 #include "tbs_kernels.cuh"
@@ -120,17 +121,25 @@ Geom make_geom(int64_t n, int64_t rb, int64_t re, int ta, int tp) {
   g.n_pad = (int)(((n + kPadAlign - 1) / kPadAlign) * kPadAlign);
   const long long I0 = g.I0, I1 = g.I1;
   g.items = (I1 - I0) * (long long)g.Mc - (long long)g.ratio * ((I1 * (I1 - 1) - I0 * (I0 - 1)) / 2);
+  g.trace = nullptr;
+  g.counter = nullptr;
+  g.chunk = 1;
   return g;
 }
 
 int pad_rows(int64_t n) { return (int)(((n + kPadAlign - 1) / kPadAlign) * kPadAlign); }
+int D_of(const tbs_args* a) { return a->dim <= 3 ? 3 : 4; }
 
 // Persistent grid for a pair-kernel instantiation: SMs x resident CTAs (at most one CTA per item).
 template <class Op, int D, class C>
 int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op& op, const uint32_t* bbox,
                 cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee) {
+  // bbox may be nulled (TBS_FORCE_CLAMP); the 64-byte block always follows the SoA copy
+  const uint32_t* bbox_block = reinterpret_cast<const uint32_t*>(soa + (size_t)D_of(a) * pad_rows(a->n));
   auto kern = pair_kernel<Op, D, C>;
-  const Geom g = make_geom(a->n, a->row_begin, a->row_end, C::TA, C::TP);
+  Geom g = make_geom(a->n, a->row_begin, a->row_end, C::TA, C::TP);
+  // work queue head: the last u64 of the 64-byte bounding-box block (zeroed per call)
+  g.counter = reinterpret_cast<unsigned long long*>(const_cast<uint32_t*>(bbox_block) + 14);
   const long long smem = ((op.smem_bytes() + 127) & ~127ll) + 2ll * D * C::TP * 4 + 16;
   if (smem > dev.smem_optin) return fail(TBS_EUNSUPPORTED, "pair kernel needs %lld B smem > %d", smem, dev.smem_optin);
   // per-instantiation cache of the attribute + occupancy query (host overhead of small calls)
@@ -152,11 +161,37 @@ int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op
   if (occ_cap > 0 && occ_cap < occ) occ = occ_cap;
   long long grid = (long long)dev.sms * occ;
   if (grid > g.items) grid = g.items;
+  g.chunk = std::max<long long>(1, g.items / (grid * 200));   // ~200 grabs per CTA
+  static const bool trace_on = getenv("TBS_TRACE") != nullptr;  // debug: CTA residency trace to stderr
+  if (trace_on) TBS_CUDA(cudaMalloc(&g.trace, (size_t)grid * 3 * 8));
   if (eb) TBS_CUDA(cudaEventRecord(eb, st));
   kern<<<(unsigned)grid, kThreads, (size_t)smem, st>>>(soa, g, op, bbox);
   TBS_CUDA(cudaGetLastError());
   g_launches.fetch_add(1);
   if (ee) TBS_CUDA(cudaEventRecord(ee, st));
+  if (trace_on) {
+    std::vector<unsigned long long> t((size_t)grid * 3);
+    TBS_CUDA(cudaStreamSynchronize(st));
+    TBS_CUDA(cudaMemcpy(t.data(), g.trace, t.size() * 8, cudaMemcpyDeviceToHost));
+    cudaFree(g.trace);
+    unsigned long long t0 = ~0ull, t1 = 0;
+    std::vector<int> per_sm(1024, 0);
+    double dmin = 1e30, dmax = 0, dsum = 0;
+    for (long long b = 0; b < grid; ++b) {
+      t0 = std::min(t0, t[3 * b + 1]);
+      t1 = std::max(t1, t[3 * b + 2]);
+      per_sm[t[3 * b] & 1023]++;
+      const double d = (double)(t[3 * b + 2] - t[3 * b + 1]);
+      dmin = std::min(dmin, d); dmax = std::max(dmax, d); dsum += d;
+    }
+    int mx = 0, mn = 1 << 30;
+    for (int k = 0; k < dev.sms; ++k) { mx = std::max(mx, per_sm[k]); mn = std::min(mn, per_sm[k]); }
+    double late = 0;  // latest CTA start relative to kernel start
+    for (long long b = 0; b < grid; ++b) late = std::max(late, (double)(t[3 * b + 1] - t0));
+    fprintf(stderr, "[tbs trace] grid %lld occ %d: CTAs/SM %d..%d, CTA time min %.3f avg %.3f max %.3f ms, "
+            "span %.3f ms, latest start %.3f ms\n", grid, occ, mn, mx, dmin * 1e-6, dsum / grid * 1e-6, dmax * 1e-6,
+            (t1 - t0) * 1e-6, late * 1e-6);
+  }
   return TBS_OK;
 }
 

@@ -52,6 +52,9 @@ struct Geom {
   int ratio;        // TA / TP
   int n_pad;        // SoA row stride (multiple of kPadAlign)
   long long items;  // total work items
+  unsigned long long* trace;  // debug only (TBS_TRACE): per CTA {smid, t_start, t_end}, else nullptr
+  unsigned long long* counter;  // work-queue head (zeroed by the loader's memset), in items
+  long long chunk;              // items grabbed per atomic
 };
 
 __device__ __forceinline__ long long items_before(const Geom& g, long long I) {
@@ -473,6 +476,8 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
   const uint32_t bar0 = smem_addr(bars), bar1 = smem_addr(bars + 1);
   const int tid = threadIdx.x;
 
+  unsigned long long t_start = 0;
+  if (g.trace != nullptr && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
   op.init(smem);
   const int variant = op.variant(bbox, D);
   if (tid == 0) {
@@ -482,21 +487,48 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
   }
   __syncthreads();
 
-  const long long beg = (g.items * (long long)blockIdx.x) / gridDim.x;
-  const long long end = (g.items * (long long)(blockIdx.x + 1)) / gridDim.x;
-  if (beg < end) {
-    int I, J;
-    item_to_tile(g, beg, I, J);
-    if (tid == 0) issue_chunk<D, C::TP>(soa, g, J, bufs, bar0);
+  // Dynamic work distribution: CTAs grab chunks of g.chunk consecutive items from a global
+  // counter, so every CTA runs until the whole triangle is done (the warp arbiter favours
+  // some CTAs of an SM over others; a static split left SMs with one straggler CTA).
+  // Thread 0 decides the NEXT item one item ahead (to prefetch its partner chunk) and
+  // publishes it through a parity-double-buffered shared slot.
+  __shared__ long long s_it[2];
+  __shared__ int s_I[2], s_J[2];
+  long long it, chunk_end = 0;
+  int I = 0, J = 0;
+  if (tid == 0) {
+    it = (long long)atomicAdd(g.counter, (unsigned long long)g.chunk);
+    if (it < g.items) {
+      chunk_end = min(it + g.chunk, g.items);
+      item_to_tile(g, it, I, J);
+      issue_chunk<D, C::TP>(soa, g, J, bufs, bar0);
+    }
+    s_it[0] = it; s_I[0] = I; s_J[0] = J;
+  }
+  __syncthreads();
+  it = s_it[0]; I = s_I[0]; J = s_J[0];
+  if (it < g.items) {
     int curI = -1;
     uint32_t phase = 0u;  // bit s = parity of buffer s
     int since = 0;
+    int s = 0;
     float2 na[D][C::KA / 2];  // negated anchor coordinates, packed (a_{2m}, a_{2m+1})
-    for (long long it = beg; it < end; ++it) {
-      const int s = (int)((it - beg) & 1);
-      int nI = I, nJ = J + 1;
-      if (nJ == g.Mc) { nI = I + 1; nJ = nI * C::RATIO; }
-      if (tid == 0 && it + 1 < end) issue_chunk<D, C::TP>(soa, g, nJ, bufs + (s ^ 1) * D * C::TP, s ? bar0 : bar1);
+    while (true) {
+      if (tid == 0) {
+        long long nit = it + 1;
+        int nI = I, nJ = J + 1;
+        if (nit < chunk_end) {
+          if (nJ == g.Mc) { nI = I + 1; nJ = nI * C::RATIO; }
+        } else {
+          nit = (long long)atomicAdd(g.counter, (unsigned long long)g.chunk);
+          if (nit < g.items) {
+            chunk_end = min(nit + g.chunk, g.items);
+            item_to_tile(g, nit, nI, nJ);
+          }
+        }
+        if (nit < g.items) issue_chunk<D, C::TP>(soa, g, nJ, bufs + (s ^ 1) * D * C::TP, s ? bar0 : bar1);
+        s_it[s ^ 1] = nit; s_I[s ^ 1] = nI; s_J[s ^ 1] = nJ;
+      }
       if (I != curI) {
         curI = I;
 #pragma unroll
@@ -536,12 +568,24 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
     item_done:
       __syncthreads();
       op.after_item(smem, since);
-      I = nI;
-      J = nJ;
+      s ^= 1;
+      it = s_it[s];
+      I = s_I[s];
+      J = s_J[s];
+      if (it >= g.items) break;
     }
   }
   __syncthreads();
   op.finish(smem);
+  if (g.trace != nullptr && tid == 0) {
+    unsigned long long t_end;
+    uint32_t smid;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    g.trace[3 * blockIdx.x] = smid;
+    g.trace[3 * blockIdx.x + 1] = t_start;
+    g.trace[3 * blockIdx.x + 2] = t_end;
+  }
 }
 
 // Sum G partial global copies into the output (one thread per bin, the paper's
