@@ -22,13 +22,13 @@ using namespace tbs;
 // Pair-engine configurations per output type: anchors/thread, partner chunk, CTAs/SM
 // (A/B-tunable with -D at build time, see tools/build_ab.py).
 #ifndef TBS_SDH_KA
-#define TBS_SDH_KA 4
+#define TBS_SDH_KA 8
 #endif
 #ifndef TBS_SDH_TP
-#define TBS_SDH_TP 512
+#define TBS_SDH_TP 1024
 #endif
 #ifndef TBS_SDH_MINB
-#define TBS_SDH_MINB 4
+#define TBS_SDH_MINB 3
 #endif
 #ifndef TBS_PCF_KA
 #define TBS_PCF_KA 8
@@ -292,6 +292,11 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
       fill(op, 4, (long long)C::KA * C::TP);
       return launch_pair<SdhSmemOp<2, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
     }
+    case 1: {
+      SdhSmemOp<1, LAT> op{};
+      fill(op, 2, (long long)C::KA * C::TP);
+      return launch_pair<SdhSmemOp<1, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+    }
     default: {
       SdhSmemOp<0, LAT> op{};
       fill(op, 1, (long long)C::KA * C::TP);
@@ -328,8 +333,11 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   const long long one_copy_budget = dev.smem_optin - 2ll * 4 * SdhCfg::TP * 4 - 256;
   if ((long long)(nb + kGuard) * 32 * 4 <= part_budget) pl.log2r = 5;
   else if ((long long)(nb + kGuard) * 4 * 4 <= part_budget) pl.log2r = 2;
+  else if ((long long)(nb + kGuard) * 2 * 4 <= one_copy_budget) pl.log2r = 1;
   else if ((long long)(nb + kGuard) * 4 <= one_copy_budget) pl.log2r = 0;
   else pl.global = true;
+  static const int r_env = [] { const char* e = getenv("TBS_LOG2R"); return e ? atoi(e) : -1; }();  // experiments
+  if (r_env >= 0 && !pl.global && (long long)(nb + kGuard) * (4ll << r_env) <= one_copy_budget) pl.log2r = r_env;
   if (a->flags & TBS_HIST_FORCE_LANE) {
     if ((long long)(nb + kGuard) * 32 * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_LANE: nb too large for smem");
     pl = SdhPlan{lattice, false, 5};
