@@ -150,13 +150,11 @@ __device__ __forceinline__ float bbox_diameter(const uint32_t* __restrict__ bbox
 // in shared memory, layout word[k * R + (lane & (R-1))]. R = 32: every lane owns a copy
 // and the 32 lanes of an ATOMS hit 32 distinct banks (no conflicts, no same-address).
 //
-// Address arithmetic on the FMA pipe, two pairs per instruction:
-//   y = RD(q * inv_w + 2^23)            FFMA2.RM: y = 2^23 + floor(q / w)       (exact)
-//   z = y + (lane_r / R - 2^23 + 2^E)   FADD2:    z = 2^E + k + lane_r / R       (exact)
-// with E = 21 - log2(R): in the binade [2^E, 2^(E+1)) one unit of k is 4R bytes of the
-// float's bit pattern, so bits(z) - bits(2^E) = 4 (k R + lane_r) is the byte offset of
-// the lane's counter. The remaining add of (smem base - bits(2^E)) is CTA-uniform and
-// folds into the ATOMS addressing mode ([R + UR]) — no integer instruction per pair.
+// Per pair: MUFU.SQRT, then for two pairs one FFMA2.RM  y = RD(q * (1/w) + 2^23) = 2^23 + k
+// (the 1/w scale and the floor in one rounding; bits(y) = bits(2^23) + k), then per pair
+// one ALU LEA.HI: (bits(y) << log2(4R)) | 4 lane_r, plus the CTA-uniform
+// (smem base - (bits(2^23) << log2(4R))) fused as a uniform-register operand — no IMAD on
+// the FMA pipe — and the ATOMS (red.shared.add.u32).
 // The clamp k <= nb-1 (one FMNMX per pair) is dropped when the loader's bounding box
 // proves k < nb + kGuard for every pair; guard rows are folded into nb-1 at the flush.
 // LATTICE: exact integer bucketing max{k : (k m)^2 <= 4^j s} for integer-valued input.
@@ -167,17 +165,13 @@ extern __shared__ __align__(128) unsigned char tbs_smem[];  // dynamic smem; his
 template <int LOG2R, bool LATTICE>
 struct SdhSmemOp {
   static constexpr int R = 1 << LOG2R;
-  static constexpr int E = 21 - LOG2R;
   int nb;             // buckets
   int rows;           // rows allocated (nb, + kGuard in float mode)
   float inv_w;        // fp32(1 / w)                       (float mode)
   float scale;        // fp32(2^j / m)                     (lattice mode)
   int m, sh;          // w = m * 2^-j, sh = 2 j            (lattice mode)
   unsigned long long* hist;  // global u64 output [nb]
-  uint32_t base;      // lattice: shared address of word 0 for this lane, minus the magic offset
-  uint32_t bmax;      // lattice: magic bits of bucket nb-1 (clamp)
-  float zc;           // float: lane_r / R - 2^23 + 2^E
-  float ymax;         // float: 2^23 + nb - 1
+  float ymax;         // float: 2^23 + nb - 1 (clamp variant)
   int flush_every;    // items between overflow flushes
 
   __host__ __device__ long long smem_bytes() const { return (long long)rows * R * 4; }
@@ -185,10 +179,6 @@ struct SdhSmemOp {
   __device__ __forceinline__ void init(unsigned char* smem) {
     uint32_t* h = reinterpret_cast<uint32_t*>(smem);
     for (int i = threadIdx.x; i < rows * R; i += kThreads) h[i] = 0u;
-    const int lane_r = threadIdx.x & (R - 1);
-    base = smem_addr(smem) + (uint32_t)(lane_r * 4) - (kMagic << (LOG2R + 2));
-    bmax = kMagic + (uint32_t)(nb - 1);
-    zc = (float)lane_r / (float)R - (kMagicF - (float)(1 << E));
     ymax = kMagicF + (float)(nb - 1);
   }
   __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
