@@ -1,0 +1,31 @@
+"""Small calls of every entry point, for compute-sanitizer (memcheck/racecheck/synccheck/initcheck)."""
+import math
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icpp_pitaksirianannt16_b200 as tbs  # noqa: E402
+import tbs_inputs as g  # noqa: E402
+
+n = int(sys.argv[1]) if len(sys.argv) > 1 else 2500
+p = torch.from_numpy(g.clustered(n, 1)).cuda()
+lat = torch.from_numpy(g.lattice(13, 2)[:n]).cuda()
+w = float(np.float32(math.sqrt(3) / 64))
+out = []
+for mode in (None, "lane", "cta", "global"):
+    out.append(tbs.sdh(p, w, 64, hist_mode=mode).sum().item())
+    out.append(tbs.sdh(lat, 0.5, 64, lattice=True, hist_mode=mode).sum().item())
+out.append(tbs.sdh(p, w, 5000).sum().item())                 # R = 4 / 2 replicas
+out.append(tbs.sdh(p, w, 64, rows=(100, 1900)).sum().item())  # row range, masked items
+out.append(tbs.sdh(p, w, 64, force_clamp=True).sum().item())
+out.append(tbs.pcf(p, 0.05).item())
+out.append(tbs.pcf(p, 0.05, rows=(7, 2000)).item())
+out.append(float(tbs.pairmatrix(p[:1001], 1.0).sum().item()))
+out.append(float(tbs.pairmatrix(p[:1000], 1.0, kernel="dist").sum().item()))
+big = torch.from_numpy(g.uniform(40000, 3)).cuda()                # main (non-small) tile config
+out.append(tbs.sdh(big, w, 64).sum().item())
+torch.cuda.synchronize()
+print("sanitize driver ok", len(out), out[:3])
