@@ -12,6 +12,8 @@ Functions and their pins (tests/test_oracle_pins.py):
   pcf            brute force, cumulative-SDH identity, cube closed form
   pairmatrix     torch.cdist float64 (library routine), symmetry, diagonal
   lattice_closed brute force of sdh_lattice on permuted lattices
+  kde            brute force (scipy pdist), closed form for coincident / two-point sets
+  rdf            hand-computed shells, uniform-cube law (g -> 1 - O(r) boundary deficit)
 Parity status: no worked example in PAPER.md prints values, so every pin is a
 mathematical one; see DESIGN.md §Oracle.
 """
@@ -57,6 +59,8 @@ def _load():
         lib.oracle_pairmatrix.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_int, ctypes.c_double, _i64, _i64,
                                           _f64p]
         lib.oracle_lattice_closed.argtypes = [_i64, _i64, ctypes.c_int, ctypes.c_int, _u64p, _i64, _u64p]
+        lib.oracle_kde.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, _i64, _i64, _f64p]
+        lib.oracle_rdf.argtypes = [_u64p, ctypes.c_int, ctypes.c_int, ctypes.c_double, _i64, ctypes.c_double, _f64p]
         lib.oracle_num_threads.restype = ctypes.c_int
         _lib = lib
     return _lib
@@ -145,3 +149,25 @@ def lattice_closed(L, m, j, nbuckets, r2=-1):
     if rc:
         raise ValueError(f"oracle_lattice_closed: status {rc}")
     return hist, int(c[0])
+
+
+def kde(points, gamma, rows=None):
+    """Gaussian kernel pair sum S = sum_{i<j} exp(-gamma d_ij^2) in float64."""
+    p, n, dim = _pts(points)
+    rb, re = _rows(rows, n)
+    out = np.zeros(1, np.float64)
+    rc = _load().oracle_kde(_ptr(p, _f32p), n, dim, float(np.float32(gamma)), rb, re, _ptr(out, _f64p))
+    if rc:
+        raise ValueError(f"oracle_kde: status {rc}")
+    return float(out[0])
+
+
+def rdf(hist, bucket_width, n, volume, dim=3):
+    """RDF g[k] = hist[k] / (C(n,2) shell_k / volume)."""
+    h = np.ascontiguousarray(hist, dtype=np.uint64)
+    g = np.zeros(len(h), np.float64)
+    rc = _load().oracle_rdf(_ptr(h, _u64p), len(h), int(dim), float(np.float32(bucket_width)), int(n), float(volume),
+                            _ptr(g, _f64p))
+    if rc:
+        raise ValueError(f"oracle_rdf: status {rc}")
+    return g

@@ -232,3 +232,40 @@ int oracle_lattice_closed(int64_t L, int64_t m, int j2, int nb, uint64_t* hist, 
   free(h2);
   return ORACLE_OK;
 }
+
+/*
+ * Kernel-density pair sum (Type-I, NEXT-2 of SURVEY §8(f); PAPER.md L303-314 names
+ * "Kernel density/regression" as a Type-I 2-BS whose per-thread output fits in
+ * registers): S = sum_{i<j} exp(-gamma * ||p_i - p_j||^2), Gaussian kernel (reading Q10's
+ * kernel). Row-range variant as above. Plain double accumulation per thread, merged.
+ */
+int oracle_kde(const float* P, int64_t n, int dim, double gamma, int64_t row_begin, int64_t row_end,
+               double* sum) {
+  if (check_common(P, n, dim, row_begin, row_end) || !isfinite(gamma) || !sum) return ORACLE_EINVAL;
+  double acc = 0.0;
+#pragma omp parallel for schedule(guided) reduction(+: acc)
+  for (int64_t i = row_begin; i < row_end; ++i)
+    for (int64_t j = i + 1; j < n; ++j) acc += exp(-gamma * dist2(P, dim, i, j));
+  *sum = acc;
+  return ORACLE_OK;
+}
+
+/*
+ * Radial distribution function (Type-II, NEXT-1; "RDF, which outputs a
+ * normalized form of SDH"): g[k] = hist[k] / ideal[k] with ideal[k] the expected count of an
+ * ideal gas of n points in volume V, ideal[k] = C(n,2) * shell_k / V and shell_k the
+ * dim-ball shell volume between k w and (k+1) w (unit-ball volumes 2, pi, 4 pi / 3, pi^2 / 2
+ * for dim 1..4). The last (clamped, open) bucket is normalised by its closed shell too.
+ */
+int oracle_rdf(const uint64_t* hist, int nb, int dim, double w, int64_t n, double volume, double* g) {
+  if (!hist || !g || nb < 1 || dim < 1 || dim > 4 || !(w > 0.0) || !(volume > 0.0) || n < 0) return ORACLE_EINVAL;
+  static const double unit_ball[5] = {0.0, 2.0, 3.14159265358979323846, 4.18879020478639098462,
+                                      4.93480220054467930942};
+  const double pairs = (double)n * (double)(n - 1) / 2.0;
+  for (int k = 0; k < nb; ++k) {
+    const double shell = unit_ball[dim] * (pow((k + 1) * w, dim) - pow(k * w, dim));
+    const double ideal = pairs * shell / volume;
+    g[k] = ideal > 0.0 ? (double)hist[k] / ideal : 0.0;
+  }
+  return ORACLE_OK;
+}

@@ -266,3 +266,36 @@ def test_pairmatrix_lattice_values():
     out = oracle.pairmatrix(p, 0.5)
     s = ((p[:, None, :].astype(np.int64) - p[None, :, :]) ** 2).sum(-1)
     np.testing.assert_allclose(out, np.exp(-0.5 * s.astype(np.float64)), rtol=1e-15, atol=0)
+
+
+# ---------------------------------------------------------------- NEXT-1 / NEXT-2: RDF and kernel-density sum
+def test_kde_bruteforce_and_closed_forms():
+    p = g.clustered(1500, 9)
+    d2 = pdist(p.astype(np.float64), "sqeuclidean")
+    for gamma in (0.0, 1.0, 50.0):
+        assert abs(oracle.kde(p, gamma) - float(np.exp(-np.float64(np.float32(gamma)) * d2).sum())) <= 1e-9 * len(d2)
+    assert oracle.kde(np.zeros((10, 3), np.float32), 3.0) == 45.0              # coincident: C(10,2) * 1
+    two = np.array([[0, 0, 0], [1, 2, 2]], np.float32)                            # d^2 = 9
+    assert abs(oracle.kde(two, 0.5) - math.exp(-4.5)) < 1e-15
+    a = oracle.kde(p, 2.0, rows=(0, 700)) + oracle.kde(p, 2.0, rows=(700, 1500))
+    assert abs(a - oracle.kde(p, 2.0)) < 1e-12 * oracle.kde(p, 2.0)
+
+
+def test_rdf_shells_and_uniform_cube():
+    h = np.array([10, 20, 30], np.uint64)
+    g3 = oracle.rdf(h, 0.5, 100, 8.0, dim=3)
+    pairs = 100 * 99 / 2
+    for k in range(3):
+        shell = 4 * math.pi / 3 * (((k + 1) * 0.5) ** 3 - (k * 0.5) ** 3)
+        assert abs(g3[k] - h[k] / (pairs * shell / 8.0)) < 1e-12
+    g1 = oracle.rdf(h, 0.5, 100, 8.0, dim=1)
+    assert abs(g1[1] - 20 / (pairs * 2 * 0.5 / 8.0)) < 1e-12
+    # uniform points in the unit cube: g(r) = P(bin) / (shell volume) -> 1 - (3/2)(r/1)*... at small r
+    p = g.uniform(4096, 1)
+    nb, w = 64, float(np.float32(math.sqrt(3) / 64))
+    hist, _ = oracle.sdh(p, w, nb)
+    gr = oracle.rdf(hist, w, 4096, 1.0)
+    expect = [(cube_cdf.F((k + 1) * w) - cube_cdf.F(k * w)) / (4 * math.pi / 3 * (((k + 1) * w) ** 3 - (k * w) ** 3))
+              for k in range(8)]
+    assert np.all(np.abs(gr[2:8] - np.array(expect[2:8])) < 0.05)             # statistical, boundary deficit
+    assert 0.85 < gr[3] < 1.0
