@@ -19,6 +19,7 @@ samples of the same workload.
 from __future__ import annotations
 
 import argparse
+import ctypes
 import json
 import math
 import os
@@ -44,6 +45,7 @@ WORKLOADS = {
     "sdh_lattice_4m": ("sdh_lattice", "lattice", 160 ** 3, 6, dict(nb=256, w=1.0)),
     "pcf_clustered_4m": ("pcf", "clustered", 1 << 22, 3, dict(r=0.03)),     # configs[2]
     "pairmatrix_64k": ("pairmatrix", "uniform", 1 << 16, 5, dict(gamma=1.0)),  # configs[4]
+    "kde_uniform_1m": ("kde", "uniform", 1 << 20, 2, dict(gamma=1.0)),        # NEXT-2 (Type-I float sum)
 }
 METRIC = "SDH pair-distances/sec (G pairs/s) at N=1M–4M, 1/2/4/8 B200, % of roofline"
 
@@ -124,6 +126,8 @@ def oracle_rate(op, p, params, rows):
         oracle.sdh_lattice(p, 1, 0, params["nb"], rows=rows)
     elif op == "pcf":
         oracle.pcf(p, params["r"], rows=rows)
+    elif op == "kde":
+        oracle.kde(p, params["gamma"], rows=rows)
     else:
         oracle.pairmatrix(p, params["gamma"], rows=rows)
     dt = time.perf_counter() - t0
@@ -224,6 +228,8 @@ def main():
         out = torch.empty(nb, dtype=torch.int64, device=dev)
     elif op == "pcf":
         out = torch.empty(1, dtype=torch.int64, device=dev)
+    elif op == "kde":
+        out = torch.empty(1, dtype=torch.float64, device=dev)
     else:
         rows_pm = (n * rank // world, n * (rank + 1) // world)
         out = torch.empty((rows_pm[1] - rows_pm[0], n), dtype=torch.float32, device=dev)
@@ -235,6 +241,8 @@ def main():
             tbs.sdh(pts, w, nb, lattice=True, out=out, events=events, group=pg)
         elif op == "pcf":
             tbs.pcf(pts, params["r"], out=out, events=events, group=pg)
+        elif op == "kde":
+            tbs.kde(pts, params["gamma"], out=out, events=events, group=pg)
         else:
             tbs.pairmatrix(pts, params["gamma"], out=out, events=events, group=pg)
 
@@ -295,6 +303,9 @@ def main():
         if op == "pcf":
             peak = pk["fp32"] / 6
             bound_note = "FP32 pipe: 6 lane-ops/pair (3 sub + 3 mul/fma)"
+        elif op == "kde":
+            peak = min(pk["fp32"] / 8, pk["mufu"])
+            bound_note = "min(FP32 pipe / 8 lane-ops per pair (distance 6, scale, sum), MUFU / 1 ex2 per pair)"
         else:
             peak = min(pk["fp32"] / 6, pk["atoms"])
             bound_note = "min(FP32 pipe / 6 lane-ops per pair, shared-atomic lanes / 1 per pair)"
@@ -302,7 +313,7 @@ def main():
                 "frac": pairs_s / peak, "peak_source": f"{bound_note}; 148 SMs x unit lanes/clk x "
                                                       f"{pk['f_max'] / 1e6:.0f} MHz (DESIGN.md §Roofline)",
                 "frac_fp32": pairs_s * 6 / pk["fp32"]}
-        if op != "pcf":
+        if op in ("sdh", "sdh_lattice"):
             roof["mufu_cap"] = pk["mufu"] / 1e9         # one MUFU.SQRT per pair: this design's ceiling
             roof["frac_of_mufu_cap"] = pairs_s / pk["mufu"]
     roof["traffic"] = None
@@ -316,14 +327,17 @@ def main():
 
     # e2e: host buffers through the public API, H2D of the points and D2H of the result each step
     e2e = None
-    if op in ("sdh", "pcf"):
+    if op in ("sdh", "pcf", "kde"):
         ph = torch.from_numpy(p_host).pin_memory()
         if world == 1:
             hh = np.zeros(nb if op == "sdh" else 1, np.uint64)
+            kh = np.zeros(1, np.float64)
 
             def e2e_step():
                 if op == "sdh":
                     tbs.sdh_host(ph.numpy(), w, nb, out=hh)
+                elif op == "kde":
+                    tbs.lib().tbs_kde(ph.numpy().ctypes.data, n, ctypes.c_float(params["gamma"]), kh.ctypes.data)
                 else:
                     tbs.pcf_host(ph.numpy(), params["r"])
         else:
@@ -333,6 +347,8 @@ def main():
                 d = ph.to(dev, non_blocking=True)
                 if op == "sdh":
                     r = tbs.sdh(d, w, nb, group=pg)
+                elif op == "kde":
+                    r = tbs.kde(d, params["gamma"], group=pg)
                 else:
                     r = tbs.pcf(d, params["r"], group=pg)
                 res_h.copy_(r)

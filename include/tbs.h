@@ -110,6 +110,20 @@ int tbs_sdh_ex(const tbs_args* args, float bucket_width, int nbuckets, uint64_t*
 int tbs_pcf_ex(const tbs_args* args, float radius, uint64_t* count);
 int tbs_pairmatrix_ex(const tbs_args* args, tbs_kernel kernel, float* out);
 
+/* ---- NEXT rows ---------------------------------------------------- */
+
+/* Kernel-density pair sum, a Type-I 2-BS ("Kernel density/regression"):
+ * *sum = sum_{i<j} exp(-gamma * ||p_i - p_j||^2) over points[n][3], host or device pointers,
+ * synchronous. fp32 kernel values, fp32 Kahan per thread, fp64 across threads; the CTA
+ * partials are combined with fp64 atomics, so the last bits can differ run to run. */
+int tbs_kde(const float* points, int64_t n, float gamma, double* sum);
+int tbs_kde_ex(const tbs_args* args, float gamma, double* sum);   /* sum: device, overwritten */
+
+/* Radial distribution function, "a normalized form of SDH": host arrays,
+ * g[k] = hist[k] / (C(n,2) * shell_k / volume), shell_k the dim-ball shell volume between
+ * k w and (k+1) w (no periodic boundary). Host-only arithmetic on an SDH result. */
+int tbs_rdf(const uint64_t* hist, int nbuckets, int dim, float bucket_width, int64_t n, double volume, double* g);
+
 /* Pair-count-balanced anchor-row partition for multi-GPU: rank r of
  * `world` gets [*row_begin, *row_end) such that sum over its rows of (n-1-i) is
  * n(n-1)/(2*world) up to one row; the ranges are disjoint and cover [0, n). Host-only. */

@@ -11,6 +11,8 @@ library or a CUDA device is missing, calls raise.
     pcf(points, radius)                   Type-I 2-point correlation count   (int64[1])
     pairmatrix(points, gamma=1.0)         Type-III Gaussian pair matrix      (float32[rows, n])
     rank_rows(n, world, rank)             pair-balanced anchor-row partition
+    kde(points, gamma)                    Type-I kernel-density pair sum      (float64[1])   (NEXT-2)
+    rdf(points, bucket_width, nb, volume) radial distribution function       (float64[nb])  (NEXT-1)
     sdh_host / pcf_host / pairmatrix_host the same through host (numpy) buffers
 """
 from __future__ import annotations
@@ -34,6 +36,7 @@ HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "
 
 # Symbols declared in include/tbs.h (checked by tests/test_abi.py).
 EXPORTS = ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
+           "tbs_kde", "tbs_kde_ex", "tbs_rdf",
            "tbs_rank_rows", "tbs_last_error", "tbs_release", "tbs_launch_count", "tbs_version")
 
 
@@ -68,13 +71,16 @@ def lib() -> ctypes.CDLL:
         L.tbs_sdh_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_float, ctypes.c_int, vp]
         L.tbs_pcf_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_float, vp]
         L.tbs_pairmatrix_ex.argtypes = [ctypes.POINTER(_Args), _Kernel, vp]
+        L.tbs_kde.argtypes = [vp, i64, ctypes.c_float, vp]
+        L.tbs_kde_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_float, vp]
+        L.tbs_rdf.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_float, i64, ctypes.c_double, vp]
         L.tbs_rank_rows.argtypes = [i64, ctypes.c_int, ctypes.c_int, ctypes.POINTER(ctypes.c_int64),
                                     ctypes.POINTER(ctypes.c_int64)]
         L.tbs_last_error.restype = ctypes.c_char_p
         L.tbs_launch_count.restype = ctypes.c_uint64
         L.tbs_release.restype = None
         for f in ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
-                  "tbs_rank_rows", "tbs_version"):
+                  "tbs_kde", "tbs_kde_ex", "tbs_rdf", "tbs_rank_rows", "tbs_version"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -175,6 +181,31 @@ def pcf(points, radius: float, *, rows=None, out=None, stream=None, events=None,
     c = out if out is not None else torch.empty(1, dtype=torch.int64, device=points.device)
     _check(lib().tbs_pcf_ex(ctypes.byref(a), float(radius), c.data_ptr()), "tbs_pcf_ex")
     return combine(c, group)
+
+
+def kde(points, gamma: float, *, rows=None, out=None, stream=None, events=None, group=None):
+    """Kernel-density pair sum (Type-I, NEXT-2): sum_{i<j} exp(-gamma d^2), float64[1] on device.
+    With a group the per-rank partial sums are combined with one all_reduce (fp64 SUM)."""
+    torch = _torch()
+    a, _ = _args(points, partition(points.shape[0], group, rows), 0, stream, events)
+    s = out if out is not None else torch.empty(1, dtype=torch.float64, device=points.device)
+    _check(lib().tbs_kde_ex(ctypes.byref(a), float(gamma), s.data_ptr()), "tbs_kde_ex")
+    return combine(s, group)
+
+
+def rdf_from_hist(hist, bucket_width: float, n: int, volume: float, dim: int = 3):
+    """RDF g[k] (NEXT-1) from an SDH histogram (host arithmetic in libtbs: tbs_rdf)."""
+    h = np.ascontiguousarray(hist.cpu().numpy() if hasattr(hist, "cpu") else hist).astype(np.uint64)
+    gr = np.empty(len(h), np.float64)
+    _check(lib().tbs_rdf(h.ctypes.data, len(h), int(dim), float(bucket_width), int(n), float(volume), gr.ctypes.data),
+           "tbs_rdf")
+    return gr
+
+
+def rdf(points, bucket_width: float, nbuckets: int, volume: float, **kw):
+    """Radial distribution function: SDH on the GPU, then the ideal-gas normalisation."""
+    h = sdh(points, bucket_width, nbuckets, **kw)
+    return rdf_from_hist(h, bucket_width, points.shape[0], volume, points.shape[1] if points.dim() > 1 else 1)
 
 
 def pairmatrix(points, gamma: float = 1.0, *, kernel: str = "gaussian", rows=None, out=None, stream=None,

@@ -410,6 +410,39 @@ int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
   return rc;
 }
 
+int kde_impl(const tbs_args* a, float gamma, double* sum) {
+  int rc = validate_common(a);
+  if (rc) return rc;
+  if (!std::isfinite(gamma)) return fail(TBS_EINVAL, "gamma must be finite");
+  if (!sum) return fail(TBS_EINVAL, "sum is NULL");
+  Device dev;
+  if ((rc = current_device(dev))) return rc;
+  cudaStream_t st = (cudaStream_t)a->stream;
+  if (a->n < 2 || a->row_begin >= a->row_end) {
+    TBS_CUDA(cudaMemsetAsync(sum, 0, 8, st));
+    return TBS_OK;
+  }
+  const int D = a->dim <= 3 ? 3 : 4;
+  float* soa = nullptr;
+  uint32_t* bbox = nullptr;
+  rc = load_points(a, D, pad_rows(a->n), &soa, reinterpret_cast<unsigned long long*>(sum), 1, st, &bbox);
+  if (!rc) {
+    KdeOp op{};
+    op.c = (float)(-(double)gamma * 1.4426950408889634);
+    op.sum = sum;
+    cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
+    const bool small = make_geom(a->n, a->row_begin, a->row_end, PcfCfg::TA, PcfCfg::TP).items < 2ll * dev.sms;
+    if (small)
+      rc = D == 3 ? launch_pair<KdeOp, 3, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee)
+                  : launch_pair<KdeOp, 4, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee);
+    else
+      rc = D == 3 ? launch_pair<KdeOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee)
+                  : launch_pair<KdeOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee);
+  }
+  if (soa) cudaFreeAsync(soa, st);
+  return rc;
+}
+
 template <int KT, int D>
 int matrix_launch(const tbs_args* a, const float* soa, int n_pad, float cexp, float* out, cudaStream_t st) {
   const int n = (int)a->n;
@@ -552,6 +585,32 @@ int tbs_pairmatrix(const float* points, int64_t n, tbs_kernel kernel, float* out
   if (n < 0 || n > TBS_MAX_N) return fail(TBS_EINVAL, "n out of range");
   return run_simple(points, n, 3, out, (size_t)n * (size_t)n * sizeof(float) + (n == 0 ? 4 : 0),
                     [&](tbs_args* a, void* o) { return pairmatrix_impl(a, kernel, (float*)o); });
+}
+
+int tbs_kde_ex(const tbs_args* args, float gamma, double* sum) {
+  g_err.clear();
+  return kde_impl(args, gamma, sum);
+}
+
+int tbs_kde(const float* points, int64_t n, float gamma, double* sum) {
+  g_err.clear();
+  return run_simple(points, n, 3, sum, 8, [&](tbs_args* a, void* out) { return kde_impl(a, gamma, (double*)out); });
+}
+
+int tbs_rdf(const uint64_t* hist, int nbuckets, int dim, float bucket_width, int64_t n, double volume, double* g) {
+  g_err.clear();
+  if (!hist || !g || nbuckets < 1 || dim < 1 || dim > 4 || !(bucket_width > 0.f) || !std::isfinite(bucket_width) ||
+      !(volume > 0.0) || !std::isfinite(volume) || n < 0)
+    return fail(TBS_EINVAL, "tbs_rdf: bad arguments");
+  static const double unit_ball[5] = {0.0, 2.0, 3.14159265358979323846, 4.18879020478639098462,
+                                      4.93480220054467930942};
+  const double w = (double)bucket_width, pairs = (double)n * (double)(n - 1) / 2.0;
+  for (int k = 0; k < nbuckets; ++k) {
+    const double shell = unit_ball[dim] * (std::pow((k + 1) * w, dim) - std::pow(k * w, dim));
+    const double ideal = pairs * shell / volume;
+    g[k] = ideal > 0.0 ? (double)hist[k] / ideal : 0.0;
+  }
+  return TBS_OK;
 }
 
 int tbs_rank_rows(int64_t n, int world, int rank, int64_t* row_begin, int64_t* row_end) {

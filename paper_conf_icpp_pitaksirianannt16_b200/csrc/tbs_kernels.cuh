@@ -299,6 +299,7 @@ struct SdhSmemOp {
       }
     }
   }
+  __device__ __forceinline__ void after_group() {}
   __device__ __forceinline__ void after_item(unsigned char* smem, int& since) {
     if (++since >= flush_every) {
       flush(smem);
@@ -353,6 +354,7 @@ struct SdhGlobalOp {
       red_gmem_inc64(p1);
     }
   }
+  __device__ __forceinline__ void after_group() {}
   __device__ __forceinline__ void after_item(unsigned char*, int&) {}
   __device__ __forceinline__ void finish(unsigned char*) {}
 };
@@ -379,6 +381,7 @@ struct PcfOp {
     }
     c += s0 + s1;
   }
+  __device__ __forceinline__ void after_group() {}
   __device__ __forceinline__ void after_item(unsigned char*, int&) {
     total += c;
     c = 0u;
@@ -396,6 +399,58 @@ struct PcfOp {
       unsigned long long s = 0;
       for (int w = 0; w < kWarps; ++w) s += red[w];
       if (s) atomicAdd(count, s);
+    }
+  }
+};
+
+// Type-I kernel-density pair sum (NEXT-2): S = sum_{i<j} exp(-gamma s). Per pair one FMUL
+// (x = -gamma log2(e) s, packed) and one MUFU.EX2; per-thread fp32 partial over one
+// partner group (4 partners x KA anchors), folded into a Kahan-compensated fp32 running sum
+// (error ~ 2u of the total), doubles from the CTA reduction on.
+struct KdeOp {
+  float c;                  // -gamma * log2(e)
+  double* sum;              // global output (zeroed by the loader)
+  float2 part;              // current group partial (two lanes of the packed pair)
+  float tot, comp;          // Kahan running sum
+  __host__ __device__ long long smem_bytes() const { return 0; }
+  __device__ __forceinline__ void init(unsigned char*) {
+    part = make_float2(0.f, 0.f);
+    tot = 0.f;
+    comp = 0.f;
+  }
+  __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
+  static constexpr int kVariants = 1;
+  __device__ __forceinline__ int variant(const uint32_t*, int) const { return 0; }
+  template <bool MASKED, int V>
+  __device__ __forceinline__ void pair2(float2 s, int pv, int a0, int a1) {
+    const float2 x = __fmul2_rn(s, make_float2(c, c));
+    float2 e = make_float2(ex2_approx(x.x), ex2_approx(x.y));
+    if (MASKED) {
+      e.x = (pv > a0) ? e.x : 0.f;
+      e.y = (pv > a1) ? e.y : 0.f;
+    }
+    part = __fadd2_rn(part, e);
+  }
+  __device__ __forceinline__ void after_group() {
+    const float y = (part.x + part.y) - comp;
+    const float t = tot + y;
+    comp = (t - tot) - y;
+    tot = t;
+    part = make_float2(0.f, 0.f);
+  }
+  __device__ __forceinline__ void after_item(unsigned char*, int&) {}
+  __device__ void finish(unsigned char* smem) {
+    double v = (double)tot - (double)comp;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+    double* red = reinterpret_cast<double*>(smem);
+    __syncthreads();
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      double t = 0.0;
+      for (int w = 0; w < kWarps; ++w) t += red[w];
+      atomicAdd(sum, t);
     }
   }
 };
@@ -453,6 +508,7 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
         op.template pair2<MASKED, V>(s, pv, MASKED ? aidx[2 * m] : 0, MASKED ? aidx[2 * m + 1] : 0);
       }
     }
+    op.after_group();
   }
 }
 

@@ -235,3 +235,52 @@ def test_launch_counter_moves(tbs):
     before = tbs.launch_count()
     sdh_gpu(tbs, g.uniform(3000, 1), 0.05, 32)
     assert tbs.launch_count() >= before + 2           # loader + pair kernel
+
+
+# ------------------------------------------------------------------ NEXT-2: kernel-density pair sum, NEXT-1: RDF
+def kde_gpu(tbs, p, gamma, **kw):
+    import torch
+    v = tbs.kde(dev(p), gamma, **kw)
+    torch.cuda.synchronize()
+    return float(v.item())
+
+
+@pytest.mark.parametrize("n", [2, 3, 1000, 2049, 5000, 30011])
+@pytest.mark.parametrize("gamma", [1.0, 100.0])
+def test_kde(tbs, n, gamma):
+    """Tolerance 1e-5 relative: ex2.approx (2 ulp) of an argument with ~3u relative error,
+    fp32 group partials of <= 32 terms, Kahan fp32 per thread, fp64 across threads."""
+    p = g.clustered(n, 40 + n)
+    ref = oracle.kde(p, gamma)
+    got = kde_gpu(tbs, p, gamma)
+    assert abs(got - ref) <= 1e-5 * abs(ref) + 1e-30, (got, ref)
+
+
+def test_kde_rows_partition_and_dims(tbs):
+    p = g.uniform(6000, 77)
+    ref = oracle.kde(p, 3.0)
+    acc = sum(kde_gpu(tbs, p, 3.0, rows=tbs.rank_rows(6000, 4, r)) for r in range(4))
+    assert abs(acc - ref) <= 1e-5 * ref
+    for dim in (1, 2, 4):
+        q = g.uniform(2500, 80 + dim, dim)
+        r = oracle.kde(q, 2.0)
+        assert abs(kde_gpu(tbs, q, 2.0) - r) <= 1e-5 * r
+    assert kde_gpu(tbs, np.zeros((0, 3), np.float32), 1.0) == 0.0
+    assert kde_gpu(tbs, np.zeros((40, 3), np.float32), 5.0) == 780.0      # C(40,2) coincident pairs
+
+
+def test_kde_host_entry_point(tbs):
+    import ctypes
+    p = g.clustered(3000, 5)
+    out = np.zeros(1, np.float64)
+    assert tbs.lib().tbs_kde(p.ctypes.data, 3000, ctypes.c_float(1.5), out.ctypes.data) == 0
+    assert abs(out[0] - oracle.kde(p, 1.5)) <= 1e-5 * out[0]
+
+
+def test_rdf(tbs):
+    p = g.uniform(20000, 3)
+    w, nb = float(np.float32(math.sqrt(3) / 128)), 128
+    h = sdh_gpu(tbs, p, w, nb)
+    gr = tbs.rdf(dev(p), w, nb, 1.0)
+    np.testing.assert_allclose(gr, oracle.rdf(h, w, 20000, 1.0), rtol=1e-13, atol=0)
+    assert 0.9 < gr[4] < 1.0        # near-ideal at small r, boundary deficit below 1
