@@ -78,6 +78,7 @@ typedef struct {
 #define TBS_HIST_FORCE_CTA 0x20u      /* SDH: one shared smem copy per CTA                 */
 #define TBS_HIST_FORCE_GLOBAL 0x40u   /* SDH: partially privatised global u64 copies       */
 #define TBS_FORCE_CLAMP 0x100u        /* SDH: never elide the nb-1 clamp (ablation/tests)   */
+#define TBS_HIST_FORCE_PASSES 0x200u  /* SDH: bucket-range passes with one smem copy (tests)   */
 
 #define TBS_MAX_N ((int64_t)1 << 30)
 #define TBS_MAX_BUCKETS (1 << 24)

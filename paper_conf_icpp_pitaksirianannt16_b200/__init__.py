@@ -31,8 +31,10 @@ TBS_HIST_FORCE_LANE = 0x10
 TBS_HIST_FORCE_CTA = 0x20
 TBS_HIST_FORCE_GLOBAL = 0x40
 TBS_FORCE_CLAMP = 0x100
+TBS_HIST_FORCE_PASSES = 0x200
 KERNELS = {"gaussian": 0, "dist2": 1, "dist": 2}
-HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "global": TBS_HIST_FORCE_GLOBAL}
+HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "global": TBS_HIST_FORCE_GLOBAL,
+              "passes": TBS_HIST_FORCE_PASSES}
 
 # Symbols declared in include/tbs.h (checked by tests/test_abi.py).
 EXPORTS = ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",

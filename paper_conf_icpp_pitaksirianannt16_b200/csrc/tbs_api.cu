@@ -60,6 +60,11 @@ using LatCfg = Cfg<TBS_LAT_CFG>;
 #define TBS_SMALL_TP 64
 #endif
 using SmallCfg = Cfg<2, TBS_SMALL_TP, 4>;
+// Use the small-problem config when the main config yields fewer than this many items per SM.
+int small_items_per_sm() {
+  static const int v = [] { const char* e = getenv("TBS_SMALL_ITEMS"); return e ? atoi(e) : 16; }();
+  return v;
+}
 
 namespace {
 
@@ -133,13 +138,15 @@ int D_of(const tbs_args* a) { return a->dim <= 3 ? 3 : 4; }
 // Persistent grid for a pair-kernel instantiation: SMs x resident CTAs (at most one CTA per item).
 template <class Op, int D, class C>
 int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op& op, const uint32_t* bbox,
-                cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee) {
+                cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee, bool first_launch_on_scratch = true) {
   // bbox may be nulled (TBS_FORCE_CLAMP); the 64-byte block always follows the SoA copy
   const uint32_t* bbox_block = reinterpret_cast<const uint32_t*>(soa + (size_t)D_of(a) * pad_rows(a->n));
   auto kern = pair_kernel<Op, D, C>;
   Geom g = make_geom(a->n, a->row_begin, a->row_end, C::TA, C::TP);
-  // work queue head: the last u64 of the 64-byte bounding-box block (zeroed per call)
+  // work queue head: the last u64 of the 64-byte bounding-box block (zeroed by the call's
+  // memset; re-zeroed here for every further launch on the same scratch, e.g. bucket passes)
   g.counter = reinterpret_cast<unsigned long long*>(const_cast<uint32_t*>(bbox_block) + 14);
+  if (!first_launch_on_scratch) TBS_CUDA(cudaMemsetAsync(g.counter, 0, sizeof(unsigned long long), st));
   const long long smem = ((op.smem_bytes() + 127) & ~127ll) + 2ll * D * C::TP * 4 + 16;
   if (smem > dev.smem_optin) return fail(TBS_EUNSUPPORTED, "pair kernel needs %lld B smem > %d", smem, dev.smem_optin);
   // per-instantiation cache of the attribute + occupancy query (host overhead of small calls)
@@ -240,6 +247,8 @@ bool dyadic(float w, long long& m, int& j) {
 struct SdhPlan {
   bool lattice, global;
   int log2r;
+  int passes = 1;       // > 1: R = 1 bucket-range passes
+  int pass_rows = 0;    // buckets per pass
 };
 
 template <int D, bool LAT>
@@ -276,7 +285,21 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
     op.flush_every = (int)std::max<long long>(1, (0xffffffffll / per_item) - 1);
   };
   using C = typename std::conditional<LAT, LatCfg, SdhCfg>::type;
-  const bool small = !LAT && make_geom(g->n, g->row_begin, g->row_end, C::TA, C::TP).items < 2ll * dev.sms;
+  const bool small =
+      !LAT && make_geom(g->n, g->row_begin, g->row_end, C::TA, C::TP).items < (long long)small_items_per_sm() * dev.sms;
+  if (pl.passes > 1) {
+    int rc = TBS_OK;
+    for (int p = 0; p < pl.passes && rc == TBS_OK; ++p) {
+      SdhSmemOp<0, LAT, true> op{};
+      fill(op, 1, (long long)C::KA * C::TP);
+      op.klo = p * pl.pass_rows;
+      const bool last = p + 1 == pl.passes;
+      op.rows = last ? (nb - op.klo) + (LAT ? 0 : kGuard) : pl.pass_rows;
+      rc = launch_pair<SdhSmemOp<0, LAT, true>, D, C>(dev, soa, g, op, bbox, st, p == 0 ? eb : nullptr,
+                                                       last ? ee : nullptr, p == 0);
+    }
+    return rc;
+  }
   switch (pl.log2r) {
     case 5: {
       SdhSmemOp<5, LAT> op{};
@@ -286,6 +309,16 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
       }
       fill(op, 32, (long long)C::KA * C::TP);
       return launch_pair<SdhSmemOp<5, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+    }
+    case 4: {
+      SdhSmemOp<4, LAT> op{};
+      fill(op, 16, (long long)C::KA * C::TP);
+      return launch_pair<SdhSmemOp<4, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+    }
+    case 3: {
+      SdhSmemOp<3, LAT> op{};
+      fill(op, 8, (long long)C::KA * C::TP);
+      return launch_pair<SdhSmemOp<3, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
     }
     case 2: {
       SdhSmemOp<2, LAT> op{};
@@ -331,13 +364,31 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   SdhPlan pl{lattice, false, 5};
   const long long part_budget = std::min<long long>(96 * 1024, dev.smem_optin - 2ll * 4 * SdhCfg::TP * 4 - 256);
   const long long one_copy_budget = dev.smem_optin - 2ll * 4 * SdhCfg::TP * 4 - 256;
-  if ((long long)(nb + kGuard) * 32 * 4 <= part_budget) pl.log2r = 5;
-  else if ((long long)(nb + kGuard) * 4 * 4 <= part_budget) pl.log2r = 2;
-  else if ((long long)(nb + kGuard) * 2 * 4 <= one_copy_budget) pl.log2r = 1;
-  else if ((long long)(nb + kGuard) * 4 <= one_copy_budget) pl.log2r = 0;
-  else pl.global = true;
+  // Measured on B200 (tools/ab_r.sh, N=1M): the most replicas that fit win even at one CTA
+  // per SM, except that R = 32 is only worth it while it leaves room for 2+ CTAs.
+  const long long rows = nb + kGuard;
+  if (rows * 32 * 4 <= part_budget) pl.log2r = 5;
+  else if (rows * 16 * 4 <= one_copy_budget) pl.log2r = 4;
+  else if (rows * 8 * 4 <= one_copy_budget) pl.log2r = 3;
+  else if (rows * 4 * 4 <= one_copy_budget) pl.log2r = 2;
+  else if (rows * 2 * 4 <= one_copy_budget) pl.log2r = 1;
+  else if (rows * 4 <= one_copy_budget) pl.log2r = 0;
+  else {
+    // beyond one copy: up to 8 bucket-range passes with one copy (each pass ~2.5e12 pairs/s
+    // vs ~0.2e12 for L2 atomics), else the partially privatised global histogram
+    const int per_pass = (int)(one_copy_budget / 4) - kGuard;
+    const int passes = (nb + per_pass - 1) / per_pass;
+    if (passes <= 8) {
+      pl.log2r = 0;
+      pl.passes = passes;
+      pl.pass_rows = per_pass;
+    } else {
+      pl.global = true;
+    }
+  }
   static const int r_env = [] { const char* e = getenv("TBS_LOG2R"); return e ? atoi(e) : -1; }();  // experiments
-  if (r_env >= 0 && !pl.global && (long long)(nb + kGuard) * (4ll << r_env) <= one_copy_budget) pl.log2r = r_env;
+  if (r_env >= 0 && !pl.global && pl.passes == 1 && (long long)(nb + kGuard) * (4ll << r_env) <= one_copy_budget)
+    pl.log2r = r_env;
   if (a->flags & TBS_HIST_FORCE_LANE) {
     if ((long long)(nb + kGuard) * 32 * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_LANE: nb too large for smem");
     pl = SdhPlan{lattice, false, 5};
@@ -345,6 +396,11 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   if (a->flags & TBS_HIST_FORCE_CTA) {
     if ((long long)(nb + kGuard) * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_CTA: nb too large for smem");
     pl = SdhPlan{lattice, false, 0};
+  }
+  if (a->flags & TBS_HIST_FORCE_PASSES) {   // bucket-range passes even when one copy fits (tests)
+    pl = SdhPlan{lattice, false, 0};
+    pl.pass_rows = std::max(1, (nb + 2) / 3);
+    pl.passes = (nb + pl.pass_rows - 1) / pl.pass_rows;
   }
   if (a->flags & TBS_HIST_FORCE_GLOBAL) pl = SdhPlan{lattice, true, 0};
 
@@ -398,7 +454,8 @@ int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
     op.r2 = (float)((double)r * (double)r);
     op.count = c;
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
-    const bool small = make_geom(a->n, a->row_begin, a->row_end, PcfCfg::TA, PcfCfg::TP).items < 2ll * dev.sms;
+    const bool small =
+        make_geom(a->n, a->row_begin, a->row_end, PcfCfg::TA, PcfCfg::TP).items < (long long)small_items_per_sm() * dev.sms;
     if (small)
       rc = D == 3 ? launch_pair<PcfOp, 3, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee)
                   : launch_pair<PcfOp, 4, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee);
@@ -431,7 +488,8 @@ int kde_impl(const tbs_args* a, float gamma, double* sum) {
     op.c = (float)(-(double)gamma * 1.4426950408889634);
     op.sum = sum;
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
-    const bool small = make_geom(a->n, a->row_begin, a->row_end, PcfCfg::TA, PcfCfg::TP).items < 2ll * dev.sms;
+    const bool small =
+        make_geom(a->n, a->row_begin, a->row_end, PcfCfg::TA, PcfCfg::TP).items < (long long)small_items_per_sm() * dev.sms;
     if (small)
       rc = D == 3 ? launch_pair<KdeOp, 3, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee)
                   : launch_pair<KdeOp, 4, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee);

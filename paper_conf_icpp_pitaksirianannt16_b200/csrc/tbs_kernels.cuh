@@ -162,9 +162,13 @@ constexpr int kGuard = 32;
 
 extern __shared__ __align__(128) unsigned char tbs_smem[];  // dynamic smem; histogram at offset 0
 
-template <int LOG2R, bool LATTICE>
+// RANGED: bucket-range pass for nb beyond one shared-memory copy: only buckets
+// [klo, klo + rows) are counted in this launch (one predicated ATOMS); the host runs
+// ceil(nb / rows) passes over the triangle instead of falling back to global atomics.
+template <int LOG2R, bool LATTICE, bool RANGED = false>
 struct SdhSmemOp {
   static constexpr int R = 1 << LOG2R;
+  int klo = 0;        // first bucket of this pass (RANGED)
   int nb;             // buckets
   int rows;           // rows allocated (nb, + kGuard in float mode)
   float inv_w;        // fp32(1 / w)                       (float mode)
@@ -245,6 +249,7 @@ struct SdhSmemOp {
   template <bool MASKED, int V>
   __device__ __forceinline__ void pair2(float2 s, int pv, int a0, int a1) {
     uint32_t ad0, ad1;
+    bool in0 = true, in1 = true;
     if (!LATTICE) {
       const float2 q = make_float2(sqrt_approx(s.x), sqrt_approx(s.y));
       float2 y = __ffma2_rd(q, make_float2(inv_w, inv_w), make_float2(kMagicF, kMagicF));
@@ -258,9 +263,13 @@ struct SdhSmemOp {
       // symbol so ptxas fuses shift + add into one ALU LEA.HI with a uniform operand.
       constexpr int S = LOG2R + 2;
       const uint32_t lo = (uint32_t)((threadIdx.x & (R - 1)) * 4) << (32 - S);
-      const uint32_t ub = smem_addr(tbs_smem) - (kMagic << S);
+      const uint32_t ub = smem_addr(tbs_smem) - ((kMagic + (RANGED ? (uint32_t)klo : 0u)) << S);
       ad0 = __funnelshift_l(lo, __float_as_uint(y.x), S) + ub;
       ad1 = __funnelshift_l(lo, __float_as_uint(y.y), S) + ub;
+      if (RANGED) {
+        in0 = __float_as_uint(y.x) - (kMagic + (uint32_t)klo) < (uint32_t)rows;
+        in1 = __float_as_uint(y.y) - (kMagic + (uint32_t)klo) < (uint32_t)rows;
+      }
     } else {
       uint32_t k0, k1;
       if (V == 0) {
@@ -269,11 +278,20 @@ struct SdhSmemOp {
         k0 = lattice_bucket<V>(s.x);
         k1 = lattice_bucket<V>(s.y);
       }
+      if (RANGED) {
+        k0 -= (uint32_t)klo;
+        k1 -= (uint32_t)klo;
+        in0 = k0 < (uint32_t)rows;
+        in1 = k1 < (uint32_t)rows;
+      }
       const uint32_t lb = smem_addr(tbs_smem) + (uint32_t)((threadIdx.x & (R - 1)) * 4);
       ad0 = (k0 << (LOG2R + 2)) + lb;
       ad1 = (k1 << (LOG2R + 2)) + lb;
     }
-    if (MASKED) {
+    if (RANGED) {
+      red_smem_inc_if(ad0, in0 && (!MASKED || pv > a0));
+      red_smem_inc_if(ad1, in1 && (!MASKED || pv > a1));
+    } else if (MASKED) {
       red_smem_inc_gt(ad0, pv, a0);
       red_smem_inc_gt(ad1, pv, a1);
     } else {
@@ -294,7 +312,7 @@ struct SdhSmemOp {
 #pragma unroll
       for (int off = 1; off < R; off <<= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
       if ((lane & (R - 1)) == 0 && v != 0ull && e < total) {
-        int k = e >> LOG2R;
+        const int k = (e >> LOG2R) + (RANGED ? klo : 0);
         atomicAdd(hist + (k < nb ? k : nb - 1), v);
       }
     }

@@ -55,6 +55,14 @@ __device__ __forceinline__ void red_smem_inc_gt(uint32_t addr, int p, int a) {
       "@q red.shared.add.u32 [%0], 1;\n}\n" ::"r"(addr),
       "r"(p), "r"(a));
 }
+// Same, predicated on a computed condition (bucket-range passes).
+__device__ __forceinline__ void red_smem_inc_if(uint32_t addr, bool c) {
+  asm volatile(
+      "{\n.reg .pred q;\n"
+      "setp.ne.s32 q, %1, 0;\n"
+      "@q red.shared.add.u32 [%0], 1;\n}\n" ::"r"(addr),
+      "r"((int)c));
+}
 // Global u64 increment (partially privatised global histogram, SASS: REDG.E.ADD.64).
 __device__ __forceinline__ void red_gmem_inc64(unsigned long long* addr) {
   asm volatile("red.global.add.u64 [%0], 1;" ::"l"(addr) : "memory");

@@ -284,3 +284,23 @@ def test_rdf(tbs):
     gr = tbs.rdf(dev(p), w, nb, 1.0)
     np.testing.assert_allclose(gr, oracle.rdf(h, w, 20000, 1.0), rtol=1e-13, atol=0)
     assert 0.9 < gr[4] < 1.0        # near-ideal at small r, boundary deficit below 1
+
+
+# ------------------------------------------------------------------ output-stage replication R and bucket-range passes
+@pytest.mark.parametrize("nb,m,j", [(700, 1, 3), (2048, 1, 5), (4096, 1, 6), (8192, 1, 7), (60000, 1, 10),
+                                    (100000, 1, 11)])
+def test_sdh_lattice_replication_and_passes(tbs, nb, m, j):
+    """nb spans R = 16, 8, 4 (one CTA copy each) and 2-3 bucket-range passes: exact."""
+    p = g.lattice(24, 9)[:9000]
+    w = m * 2.0 ** -j
+    h = sdh_gpu(tbs, p, w, nb, lattice=True)
+    assert h.tolist() == oracle.sdh_lattice(p, m, j, nb).tolist()
+
+
+@pytest.mark.parametrize("nb", [64, 1000, 70000])
+def test_sdh_forced_passes_float(tbs, nb):
+    p = g.clustered(7000, 12)
+    w = float(np.float32(math.sqrt(3) / min(nb, 4000)))
+    h = sdh_gpu(tbs, p, w, nb, hist_mode="passes" if nb < 50000 else None)
+    ho, amb = oracle.sdh(p, w, nb)
+    check_sdh_float(h, ho, amb)
