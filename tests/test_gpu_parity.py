@@ -304,3 +304,32 @@ def test_sdh_forced_passes_float(tbs, nb):
     h = sdh_gpu(tbs, p, w, nb, hist_mode="passes" if nb < 50000 else None)
     ho, amb = oracle.sdh(p, w, nb)
     check_sdh_float(h, ho, amb)
+
+
+# ------------------------------------------------------------------ CUDA-graph capture of the stream-ordered API
+def test_cuda_graph_capture_replay(tbs):
+    """tbs_*_ex enqueue only stream-ordered work (cudaMallocAsync scratch, memset, kernels,
+    cudaFreeAsync), so a call can be captured once and replayed; replays recompute from the
+    (possibly updated) input buffer."""
+    import torch
+    p = dev(g.clustered(9000, 8))
+    w = float(np.float32(math.sqrt(3) / 256))
+    h = torch.empty(256, dtype=torch.int64, device="cuda")
+    c = torch.empty(1, dtype=torch.int64, device="cuda")
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        tbs.sdh(p, w, 256, out=h)              # warm-up outside capture (occupancy cache, attributes)
+        tbs.pcf(p, 0.03, out=c)
+    torch.cuda.synchronize()
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph, stream=s):
+        tbs.sdh(p, w, 256, out=h)
+        tbs.pcf(p, 0.03, out=c)
+    for seed in (8, 9):
+        p.copy_(torch.from_numpy(g.clustered(9000, seed)))
+        graph.replay()
+        torch.cuda.synchronize()
+        ho, amb = oracle.sdh(p.cpu().numpy(), w, 256)
+        check_sdh_float(h.cpu().numpy(), ho, amb)
+        co, ca = oracle.pcf(p.cpu().numpy(), 0.03)
+        check_pcf_float(int(c.item()), co, ca)
