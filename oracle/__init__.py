@@ -14,6 +14,7 @@ Functions and their pins (tests/test_oracle_pins.py):
   lattice_closed brute force of sdh_lattice on permuted lattices
   kde            brute force (scipy pdist), closed form for coincident / two-point sets
   rdf            hand-computed shells, uniform-cube law (g -> 1 - O(r) boundary deficit)
+  pairmatrix_hd  torch.cdist float64 on the decoded bf16 features, symmetry, diagonal
 Parity status: no worked example in PAPER.md prints values, so every pin is a
 mathematical one; see DESIGN.md §Oracle.
 """
@@ -61,6 +62,8 @@ def _load():
         lib.oracle_lattice_closed.argtypes = [_i64, _i64, ctypes.c_int, ctypes.c_int, _u64p, _i64, _u64p]
         lib.oracle_kde.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, _i64, _i64, _f64p]
         lib.oracle_rdf.argtypes = [_u64p, ctypes.c_int, ctypes.c_int, ctypes.c_double, _i64, ctypes.c_double, _f64p]
+        lib.oracle_pairmatrix_hd.argtypes = [ctypes.POINTER(ctypes.c_uint16), _i64, ctypes.c_int, ctypes.c_int,
+                                             ctypes.c_double, _i64, _i64, _f64p]
         lib.oracle_num_threads.restype = ctypes.c_int
         _lib = lib
     return _lib
@@ -171,3 +174,16 @@ def rdf(hist, bucket_width, n, volume, dim=3):
     if rc:
         raise ValueError(f"oracle_rdf: status {rc}")
     return g
+
+
+def pairmatrix_hd(features_bf16_bits, gamma, rows=None, ktype=0):
+    """High-dimensional pair matrix from bf16 features given as uint16 bit patterns [n][d]."""
+    x = np.ascontiguousarray(features_bf16_bits, dtype=np.uint16)
+    n, d = x.shape
+    rb, re = _rows(rows, n)
+    out = np.zeros((re - rb, n), np.float64)
+    rc = _load().oracle_pairmatrix_hd(x.ctypes.data_as(ctypes.POINTER(ctypes.c_uint16)), n, d, int(ktype),
+                                      float(np.float32(gamma)), rb, re, _ptr(out, _f64p))
+    if rc:
+        raise ValueError(f"oracle_pairmatrix_hd: status {rc}")
+    return out

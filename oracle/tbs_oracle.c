@@ -269,3 +269,37 @@ int oracle_rdf(const uint64_t* hist, int nb, int dim, double w, int64_t n, doubl
   }
   return ORACLE_OK;
 }
+
+/* bf16 bit pattern -> float (exact: bf16 is the top half of an fp32). */
+static double bf16_to_double(uint16_t h) {
+  uint32_t u = (uint32_t)h << 16;
+  float f;
+  memcpy(&f, &u, 4);
+  return (double)f;
+}
+
+/*
+ * High-dimensional Type-III pair matrix (NEXT-3 of SURVEY §8(f); "Kernel
+ * methods which compute kernel functions for all pairs of data in the feature space"):
+ * features are bf16 [n][d] row-major (passed as their 16-bit patterns);
+ * out[(i - row_begin) * n + j] = K(x_i, x_j) for i in [row_begin, row_end), j in [0, n), with
+ * K as in oracle_pairmatrix (0 Gaussian exp(-gamma s), 1 s, 2 sqrt(s)), s = ||x_i - x_j||^2
+ * evaluated directly (difference, then square) in double.
+ */
+int oracle_pairmatrix_hd(const uint16_t* X, int64_t n, int d, int ktype, double gamma, int64_t row_begin,
+                         int64_t row_end, double* out) {
+  if (n < 0 || d < 1 || row_begin < 0 || row_end < row_begin || row_end > n || ktype < 0 || ktype > 2 ||
+      !isfinite(gamma) || (n > 0 && !X) || (row_end > row_begin && !out))
+    return ORACLE_EINVAL;
+#pragma omp parallel for schedule(guided)
+  for (int64_t i = row_begin; i < row_end; ++i)
+    for (int64_t j = 0; j < n; ++j) {
+      double s = 0.0;
+      for (int c = 0; c < d; ++c) {
+        const double t = bf16_to_double(X[i * d + c]) - bf16_to_double(X[j * d + c]);
+        s += t * t;
+      }
+      out[(i - row_begin) * n + j] = ktype == 0 ? exp(-gamma * s) : ktype == 1 ? s : sqrt(s);
+    }
+  return ORACLE_OK;
+}

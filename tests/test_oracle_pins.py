@@ -299,3 +299,27 @@ def test_rdf_shells_and_uniform_cube():
               for k in range(8)]
     assert np.all(np.abs(gr[2:8] - np.array(expect[2:8])) < 0.05)             # statistical, boundary deficit
     assert 0.85 < gr[3] < 1.0
+
+
+# ---------------------------------------------------------------- NEXT-3: high-dimensional Type-III (bf16 features)
+def bf16_bits(a):
+    """Round-to-nearest-even fp32 -> bf16 bit patterns (test-side input construction)."""
+    u = np.ascontiguousarray(a, dtype=np.float32).view(np.uint32).astype(np.uint64)
+    r = ((u >> 16) & 1) + 0x7FFF
+    return ((u + r) >> 16).astype(np.uint16)
+
+
+def test_pairmatrix_hd_vs_cdist():
+    import torch
+    rng = np.random.default_rng(3)
+    x = bf16_bits(rng.standard_normal((300, 40)).astype(np.float32))
+    xf = (x.astype(np.uint32) << 16).view(np.float32).astype(np.float64)
+    t = torch.from_numpy(xf)
+    d = torch.cdist(t, t, compute_mode="donot_use_mm_for_euclid_dist").numpy()
+    np.testing.assert_allclose(oracle.pairmatrix_hd(x, 0.05), np.exp(-np.float64(np.float32(0.05)) * d * d),
+                               rtol=1e-12, atol=0)
+    np.testing.assert_allclose(oracle.pairmatrix_hd(x, 0.0, ktype=1), d * d, rtol=1e-12, atol=1e-12)
+    np.testing.assert_allclose(oracle.pairmatrix_hd(x, 0.0, ktype=2), d, rtol=1e-12, atol=1e-12)
+    full = oracle.pairmatrix_hd(x, 0.3)
+    assert np.array_equal(full, full.T) and np.all(np.diag(full) == 1.0)
+    assert np.array_equal(oracle.pairmatrix_hd(x, 0.3, rows=(17, 90)), full[17:90])
