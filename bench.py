@@ -46,6 +46,7 @@ WORKLOADS = {
     "pcf_clustered_4m": ("pcf", "clustered", 1 << 22, 3, dict(r=0.03)),     # configs[2]
     "pairmatrix_64k": ("pairmatrix", "uniform", 1 << 16, 5, dict(gamma=1.0)),  # configs[4]
     "kde_uniform_1m": ("kde", "uniform", 1 << 20, 2, dict(gamma=1.0)),        # NEXT-2 (Type-I float sum)
+    "pairmatrix_hd_64k_d64": ("pairmatrix_hd", "uniform", 1 << 16, 7, dict(d=64, gamma=1.0 / 64)),  # NEXT-3
 }
 METRIC = "SDH pair-distances/sec (G pairs/s) at N=1M–4M, 1/2/4/8 B200, % of roofline"
 
@@ -128,31 +129,39 @@ def oracle_rate(op, p, params, rows):
         oracle.pcf(p, params["r"], rows=rows)
     elif op == "kde":
         oracle.kde(p, params["gamma"], rows=rows)
+    elif op == "pairmatrix_hd":
+        oracle.pairmatrix_hd(bf16_bits(p), params["gamma"], rows=rows)
     else:
         oracle.pairmatrix(p, params["gamma"], rows=rows)
     dt = time.perf_counter() - t0
     b, e = rows
-    units = (e - b) * n if op == "pairmatrix" else (e - b) * (2 * n - b - e - 1) // 2
+    units = (e - b) * n if op.startswith("pairmatrix") else (e - b) * (2 * n - b - e - 1) // 2
     return units, dt
+
+
+def bf16_bits(a):
+    """fp32 -> bf16 (round to nearest even) bit patterns, the same rounding torch applies."""
+    u = np.ascontiguousarray(a, dtype=np.float32).view(np.uint32).astype(np.uint64)
+    return ((u + ((u >> np.uint64(16)) & np.uint64(1)) + np.uint64(0x7FFF)) >> np.uint64(16)).astype(np.uint16)
 
 
 def sample_rows(op, n, target_units):
     """Anchor rows [0, R) holding about target_units pairs (matrix: entries)."""
-    per = n if op == "pairmatrix" else max(n - 1, 1)
+    per = n if op.startswith("pairmatrix") else max(n - 1, 1)
     return (0, int(min(n, max(1, target_units // per))))
 
 
 def cpu_baseline(op, p, params, seconds):
     import oracle
     n = p.shape[0]
-    u, dt = oracle_rate(op, p, params, sample_rows(op, n, 2e8 if op != "pairmatrix" else 2e7))
+    u, dt = oracle_rate(op, p, params, sample_rows(op, n, 2e8 if not op.startswith("pairmatrix") else 2e7))
     rate = u / dt
     rows = sample_rows(op, n, rate * seconds)
     u, dt = oracle_rate(op, p, params, rows)
-    return dict(value=u / dt / 1e9, unit="G pairs/s" if op != "pairmatrix" else "G entries/s",
+    return dict(value=u / dt / 1e9, unit="G pairs/s" if not op.startswith("pairmatrix") else "G entries/s",
                 cores=oracle.num_threads(), kind="oracle",
                 sample=f"anchor rows [{rows[0]},{rows[1]}) of the same N={n} input ({u:.3e} "
-                       f"{'pairs' if op != 'pairmatrix' else 'entries'}, {dt:.1f} s, fp64, OpenMP)")
+                       f"{'pairs' if not op.startswith('pairmatrix') else 'entries'}, {dt:.1f} s, fp64, OpenMP)")
 
 
 def run_reference(args, wl):
@@ -160,12 +169,12 @@ def run_reference(args, wl):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    p = gen.make(dist_, n, seed)
-    unit = "G pairs/s" if op != "pairmatrix" else "G entries/s"
+    p = gen.make(dist_, n, seed, params.get("d", 3))
+    unit = "G pairs/s" if not op.startswith("pairmatrix") else "G entries/s"
     import oracle
     # each step: a bounded anchor-row sample, sized for ~120 s over the whole run
     per_step = max(2.0, 120.0 / max(1, args.steps + args.warmup))
-    u0, dt0 = oracle_rate(op, p, params, sample_rows(op, n, 2e8 if op != "pairmatrix" else 2e7))
+    u0, dt0 = oracle_rate(op, p, params, sample_rows(op, n, 2e8 if not op.startswith("pairmatrix") else 2e7))
     rows = sample_rows(op, n, u0 / dt0 * per_step)
     for _ in range(args.warmup):
         oracle_rate(op, p, params, rows)
@@ -217,8 +226,10 @@ def main():
         pg = dist.group.WORLD
 
     op, dist_, n, seed, params = WORKLOADS[wl]
-    p_host = gen.make(dist_, n, seed)
+    p_host = gen.make(dist_, n, seed, params.get("d", 3))
     pts = torch.from_numpy(p_host).to(dev)
+    if op == "pairmatrix_hd":
+        pts = pts.to(torch.bfloat16)        # the API's feature type (input construction, untimed)
     st = torch.cuda.current_stream(dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     nb = params.get("nb", 1)
@@ -243,6 +254,8 @@ def main():
             tbs.pcf(pts, params["r"], out=out, events=events, group=pg)
         elif op == "kde":
             tbs.kde(pts, params["gamma"], out=out, events=events, group=pg)
+        elif op == "pairmatrix_hd":
+            tbs.pairmatrix_hd(pts, params["gamma"], out=out, events=events, group=pg)
         else:
             tbs.pairmatrix(pts, params["gamma"], out=out, events=events, group=pg)
 
@@ -283,12 +296,13 @@ def main():
     else:
         kavg = sum(kms) / len(kms)
 
-    units = units_of("pairmatrix" if op == "pairmatrix" else "sdh", n)
+    is_matrix = op in ("pairmatrix", "pairmatrix_hd")
+    units = units_of("pairmatrix" if is_matrix else "sdh", n)
     value = units * args.steps / (ms * 1e-3) / 1e9
-    unit = "G pairs/s" if op != "pairmatrix" else "G entries/s"
+    unit = "G pairs/s" if not is_matrix else "G entries/s"
     pk = peaks()
     # dominant kernel (pair kernel / matrix kernel) on this rank: its share of the units
-    if op == "pairmatrix":
+    if is_matrix:
         rows_pm = (n * rank // world, n * (rank + 1) // world)
         rank_units = (rows_pm[1] - rows_pm[0]) * n
         bytes_ = rank_units * 4.0

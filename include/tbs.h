@@ -125,6 +125,18 @@ int tbs_kde_ex(const tbs_args* args, float gamma, double* sum);   /* sum: device
  * k w and (k+1) w (no periodic boundary). Host-only arithmetic on an SDH result. */
 int tbs_rdf(const uint64_t* hist, int nbuckets, int dim, float bucket_width, int64_t n, double volume, double* g);
 
+/* High-dimensional Type-III pair matrix on the 5th-generation tensor cores (NEXT-3;
+ * PAPER.md L330-332 kernel methods over feature spaces): features are bf16 [n][d] row-major
+ * (raw 16-bit patterns), 1 <= d <= 128 (larger d: TBS_EUNSUPPORTED). out[i*n + j] = K(x_i, x_j)
+ * in fp32 for all i, j (diagonal included) with s = |x_i|^2 + |x_j|^2 - 2 x_i.x_j from
+ * tcgen05 bf16 x bf16 -> fp32 dot products (error ~2^-22 (|x_i|^2 + |x_j|^2) on s), clamped
+ * at 0 for the distance kernels. Host or device pointers, synchronous. */
+int tbs_pairmatrix_hd(const uint16_t* features, int64_t n, int d, tbs_kernel kernel, float* out);
+/* Device pointers, rows [row_begin, row_end) x n into out, enqueued on `stream`; optional
+ * cudaEvent_t pair recorded around the tensor-core kernel. */
+int tbs_pairmatrix_hd_ex(const uint16_t* features, int64_t n, int d, int64_t row_begin, int64_t row_end,
+                         tbs_kernel kernel, float* out, void* stream, void* ev_begin, void* ev_end);
+
 /* Pair-count-balanced anchor-row partition for multi-GPU: rank r of
  * `world` gets [*row_begin, *row_end) such that sum over its rows of (n-1-i) is
  * n(n-1)/(2*world) up to one row; the ranges are disjoint and cover [0, n). Host-only. */

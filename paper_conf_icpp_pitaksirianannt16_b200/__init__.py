@@ -38,7 +38,7 @@ HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "
 
 # Symbols declared in include/tbs.h (checked by tests/test_abi.py).
 EXPORTS = ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
-           "tbs_kde", "tbs_kde_ex", "tbs_rdf",
+           "tbs_kde", "tbs_kde_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex",
            "tbs_rank_rows", "tbs_last_error", "tbs_release", "tbs_launch_count", "tbs_version")
 
 
@@ -76,13 +76,15 @@ def lib() -> ctypes.CDLL:
         L.tbs_kde.argtypes = [vp, i64, ctypes.c_float, vp]
         L.tbs_kde_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_float, vp]
         L.tbs_rdf.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_float, i64, ctypes.c_double, vp]
+        L.tbs_pairmatrix_hd.argtypes = [vp, i64, ctypes.c_int, _Kernel, vp]
+        L.tbs_pairmatrix_hd_ex.argtypes = [vp, i64, ctypes.c_int, i64, i64, _Kernel, vp, vp, vp, vp]
         L.tbs_rank_rows.argtypes = [i64, ctypes.c_int, ctypes.c_int, ctypes.POINTER(ctypes.c_int64),
                                     ctypes.POINTER(ctypes.c_int64)]
         L.tbs_last_error.restype = ctypes.c_char_p
         L.tbs_launch_count.restype = ctypes.c_uint64
         L.tbs_release.restype = None
         for f in ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
-                  "tbs_kde", "tbs_kde_ex", "tbs_rdf", "tbs_rank_rows", "tbs_version"):
+                  "tbs_kde", "tbs_kde_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex", "tbs_rank_rows", "tbs_version"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -225,6 +227,28 @@ def pairmatrix(points, gamma: float = 1.0, *, kernel: str = "gaussian", rows=Non
     o = out if out is not None else torch.empty((nr, n), dtype=torch.float32, device=points.device)
     _check(lib().tbs_pairmatrix_ex(ctypes.byref(a), _Kernel(KERNELS[kernel], float(gamma)), o.data_ptr()),
            "tbs_pairmatrix_ex")
+    return o
+
+
+def pairmatrix_hd(features, gamma: float = 1.0, *, kernel: str = "gaussian", rows=None, out=None, stream=None,
+                  events=None, group=None):
+    """High-dimensional Type-III pair matrix on the tensor cores (NEXT-3): features is a CUDA
+    bfloat16 tensor [n, d] (d <= 128); returns float32 rows [b, e) x n."""
+    torch = _torch()
+    if not (isinstance(features, torch.Tensor) and features.is_cuda and features.dtype == torch.bfloat16):
+        raise TypeError("features must be a CUDA bfloat16 tensor [n, d]")
+    x = features.contiguous()
+    n, d = x.shape
+    if group is not None:
+        import torch.distributed as dist
+        W, r = dist.get_world_size(group), dist.get_rank(group)
+        rows = (n * r // W, n * (r + 1) // W)
+    rb, re = (0, n) if rows is None else (int(rows[0]), int(rows[1]))
+    st = stream if stream is not None else torch.cuda.current_stream(x.device)
+    o = out if out is not None else torch.empty((re - rb, n), dtype=torch.float32, device=x.device)
+    ev = (events[0].cuda_event, events[1].cuda_event) if events is not None else (None, None)
+    _check(lib().tbs_pairmatrix_hd_ex(x.data_ptr(), n, d, rb, re, _Kernel(KERNELS[kernel], float(gamma)), o.data_ptr(),
+                                      st.cuda_stream, ev[0], ev[1]), "tbs_pairmatrix_hd_ex")
     return o
 
 

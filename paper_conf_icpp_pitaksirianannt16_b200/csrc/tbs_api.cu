@@ -1,6 +1,7 @@
 // tbs_api.cu — the C-ABI host library (libtbs.so): argument validation, output-stage
 // selection, stream-ordered scratch, the work geometry, launches. Declared in
 // include/tbs.h (which cites the paper passages defining each operation).
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -16,6 +17,7 @@
 
 #include "tbs.h"
 #include "tbs_kernels.cuh"
+#include "tbs_hd.cuh"
 
 using namespace tbs;
 
@@ -544,6 +546,90 @@ int pairmatrix_impl(const tbs_args* a, tbs_kernel k, float* out) {
   return rc;
 }
 
+// ---- NEXT-3: high-dimensional Type-III on tcgen05 ---------------------------------------
+using EncodeTiledFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+int encode_tiled_fn(EncodeTiledFn& fn) {
+  static EncodeTiledFn cached = nullptr;
+  if (!cached) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    TBS_CUDA(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q));
+    if (!p || q != cudaDriverEntryPointSuccess) return fail(TBS_ECUDA, "cuTensorMapEncodeTiled unavailable");
+    cached = reinterpret_cast<EncodeTiledFn>(p);
+  }
+  fn = cached;
+  return TBS_OK;
+}
+
+int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_kernel k, float* out, cudaStream_t st,
+            cudaEvent_t eb, cudaEvent_t ee) {
+  if (n < 0 || n > (1 << 24)) return fail(TBS_EINVAL, "n out of range for the pair matrix");
+  if (d < 1) return fail(TBS_EINVAL, "d must be >= 1");
+  if (d > hd::kKBlock * hd::kMaxKBlocks) return fail(TBS_EUNSUPPORTED, "d > 128 not supported yet");
+  if (rb < 0 || re < rb || re > n) return fail(TBS_EINVAL, "row range outside [0, n]");
+  if (k.type < 0 || k.type > 2) return fail(TBS_EINVAL, "kernel type %d unknown", k.type);
+  if (k.type == TBS_K_GAUSSIAN && !std::isfinite(k.gamma)) return fail(TBS_EINVAL, "gamma must be finite");
+  if (re > rb && (!x || !out)) return fail(TBS_EINVAL, "NULL features or output");
+  if (re == rb) return TBS_OK;
+  Device dev;
+  int rc = current_device(dev);
+  if (rc) return rc;
+  const int dp = d <= hd::kKBlock ? hd::kKBlock : 2 * hd::kKBlock;
+  const int64_t n_pad = (n + hd::kTile - 1) / hd::kTile * hd::kTile;
+  unsigned char* scratch = nullptr;
+  const size_t xbytes = (size_t)n_pad * dp * 2;
+  TBS_CUDA(cudaMallocAsync((void**)&scratch, xbytes + (size_t)n_pad * 4, st));
+  uint16_t* xp = reinterpret_cast<uint16_t*>(scratch);
+  float* norms = reinterpret_cast<float*>(scratch + xbytes);
+  {
+    const int threads = 256;
+    const long long blocks = std::min<long long>((n_pad * 32 + threads - 1) / threads, (long long)dev.sms * 16);
+    hd::hd_prep<<<(unsigned)blocks, threads, 0, st>>>(x, (int)n, d, (int)n_pad, dp, xp, norms);
+    rc = cudaGetLastError() == cudaSuccess ? TBS_OK : fail(TBS_ECUDA, "hd_prep launch failed");
+    g_launches.fetch_add(1);
+  }
+  EncodeTiledFn enc = nullptr;
+  if (!rc) rc = encode_tiled_fn(enc);
+  CUtensorMap tmap;
+  if (!rc) {
+    const cuuint64_t dims[2] = {(cuuint64_t)dp, (cuuint64_t)n_pad};
+    const cuuint64_t strides[1] = {(cuuint64_t)dp * 2};
+    const cuuint32_t box[2] = {(cuuint32_t)hd::kKBlock, (cuuint32_t)hd::kTile};
+    const cuuint32_t estr[2] = {1, 1};
+    const CUresult cr = enc(&tmap, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, xp, dims, strides, box, estr,
+                            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (cr != CUDA_SUCCESS) rc = fail(TBS_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)cr);
+  }
+  if (!rc) {
+    const int I0 = (int)(rb / hd::kTile), I1 = (int)((re + hd::kTile - 1) / hd::kTile);
+    const int tiles_i = I1 - I0, tiles_j = (int)(n_pad / hd::kTile);
+    const long long ntiles = (long long)tiles_i * tiles_j;
+    const int grid = (int)std::min<long long>(ntiles, dev.sms);
+    const int smem = hd::Smem::BYTES + 1024;
+    const float cexp = (float)(-(double)k.gamma * 1.4426950408889634);
+    const int kblocks = dp / hd::kKBlock;
+    auto launch = [&](auto kern) -> int {
+      TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+      if (eb) TBS_CUDA(cudaEventRecord(eb, st));
+      kern<<<grid, hd::kThreads, smem, st>>>(tmap, norms, (int)n, kblocks, I0, tiles_i, tiles_j, (int)rb, (int)re,
+                                             cexp, out);
+      TBS_CUDA(cudaGetLastError());
+      g_launches.fetch_add(1);
+      if (ee) TBS_CUDA(cudaEventRecord(ee, st));
+      return TBS_OK;
+    };
+    rc = k.type == 0 ? launch(hd::hd_pairmatrix_kernel<0>)
+         : k.type == 1 ? launch(hd::hd_pairmatrix_kernel<1>)
+                       : launch(hd::hd_pairmatrix_kernel<2>);
+  }
+  cudaFreeAsync(scratch, st);
+  return rc;
+}
+
 // ---- host-or-device simple entry points ------------------------------------------
 int is_device_ptr(const void* p, bool& dev) {
   dev = false;
@@ -669,6 +755,49 @@ int tbs_rdf(const uint64_t* hist, int nbuckets, int dim, float bucket_width, int
     g[k] = ideal > 0.0 ? (double)hist[k] / ideal : 0.0;
   }
   return TBS_OK;
+}
+
+int tbs_pairmatrix_hd_ex(const uint16_t* features, int64_t n, int d, int64_t row_begin, int64_t row_end,
+                         tbs_kernel kernel, float* out, void* stream, void* ev_begin, void* ev_end) {
+  g_err.clear();
+  return hd_impl(features, n, d, row_begin, row_end, kernel, out, (cudaStream_t)stream, (cudaEvent_t)ev_begin,
+                 (cudaEvent_t)ev_end);
+}
+
+int tbs_pairmatrix_hd(const uint16_t* features, int64_t n, int d, tbs_kernel kernel, float* out) {
+  g_err.clear();
+  if (n < 0 || d < 1 || !out || (n > 0 && !features)) return fail(TBS_EINVAL, "tbs_pairmatrix_hd: bad arguments");
+  bool fdev = false, odev = false;
+  is_device_ptr(features, fdev);
+  is_device_ptr(out, odev);
+  if (n > 0 && fdev != odev) return fail(TBS_EINVAL, "features and out must both be host or both device pointers");
+  cudaStream_t st = cudaStreamPerThread;
+  if (odev) {
+    int rc = hd_impl(features, n, d, 0, n, kernel, out, st, nullptr, nullptr);
+    if (!rc) TBS_CUDA(cudaStreamSynchronize(st));
+    return rc;
+  }
+  uint16_t* df = nullptr;
+  float* dout = nullptr;
+  const size_t fb = (size_t)n * d * 2, ob = (size_t)n * n * 4;
+  if (fb) TBS_CUDA(cudaMallocAsync((void**)&df, fb, st));
+  cudaError_t e = cudaMallocAsync((void**)&dout, ob ? ob : 4, st);
+  if (e != cudaSuccess) {
+    if (df) cudaFreeAsync(df, st);
+    return fail(TBS_ENOMEM, "cudaMallocAsync(%zu): %s", ob, cudaGetErrorString(e));
+  }
+  if (fb) e = cudaMemcpyAsync(df, features, fb, cudaMemcpyHostToDevice, st);
+  int rc = e != cudaSuccess ? fail(TBS_ECUDA, "H2D: %s", cudaGetErrorString(e))
+                            : hd_impl(df, n, d, 0, n, kernel, dout, st, nullptr, nullptr);
+  if (!rc && ob) {
+    e = cudaMemcpyAsync(out, dout, ob, cudaMemcpyDeviceToHost, st);
+    if (e != cudaSuccess) rc = fail(TBS_ECUDA, "D2H: %s", cudaGetErrorString(e));
+  }
+  if (df) cudaFreeAsync(df, st);
+  cudaFreeAsync(dout, st);
+  e = cudaStreamSynchronize(st);
+  if (!rc && e != cudaSuccess) rc = fail(TBS_ECUDA, "sync: %s", cudaGetErrorString(e));
+  return rc;
 }
 
 int tbs_rank_rows(int64_t n, int world, int rank, int64_t* row_begin, int64_t* row_end) {

@@ -166,3 +166,24 @@ def test_pairmatrix_64k_sampled_rows(tbs):
     for k, r in enumerate(rows):
         ref = oracle.pairmatrix(p, 1.0, rows=(r, r + 1))[0]
         check_matrix(got[k], ref)
+
+
+# ---------------------------------------------------------------- NEXT-3 at full size: N=64K, d=64 (17.2 GB fp32)
+def test_pairmatrix_hd_64k_sampled_rows(tbs):
+    import torch
+    n, d = 1 << 16, 64
+    x = torch.from_numpy(g.uniform(n, 7, d)).cuda().to(torch.bfloat16)
+    xb = x.view(torch.int16).cpu().numpy().view(np.uint16)
+    out = tbs.pairmatrix_hd(x, 1.0 / d)
+    rng = np.random.default_rng(1)
+    rows = sorted(set([0, n - 1] + rng.integers(0, n, 62).tolist()))
+    got = host(out.index_select(0, torch.tensor(rows, device=out.device))).astype(np.float64)
+    del out
+    torch.cuda.empty_cache()
+    xf = (xb.astype(np.uint32) << 16).view(np.float32).astype(np.float64)
+    nrm = (xf * xf).sum(1)
+    g32 = np.float64(np.float32(1.0 / d))
+    for k, r in enumerate(rows):
+        ref = oracle.pairmatrix_hd(xb, 1.0 / d, rows=(r, r + 1))[0]
+        B = 2.0 ** -20 * (nrm[r] + nrm + 2 * np.abs(xf) @ np.abs(xf[r]))
+        assert np.all(np.abs(got[k] - ref) <= ref * (g32 * B + 2e-6)), r

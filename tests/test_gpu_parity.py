@@ -333,3 +333,55 @@ def test_cuda_graph_capture_replay(tbs):
         check_sdh_float(h.cpu().numpy(), ho, amb)
         co, ca = oracle.pcf(p.cpu().numpy(), 0.03)
         check_pcf_float(int(c.item()), co, ca)
+
+
+# ------------------------------------------------------------------ NEXT-3: high-dimensional Type-III on tcgen05
+def _bf16_bits(a):
+    u = np.ascontiguousarray(a, dtype=np.float32).view(np.uint32).astype(np.uint64)
+    return ((u + ((u >> 16) & 1) + 0x7FFF) >> 16).astype(np.uint16)
+
+
+def _hd_bound(xbits):
+    """Per-entry bound on |s_gpu - s|: fp32 norms and fp32 tensor-core accumulation
+    of exact bf16 products, 2^-20 (|x_i|^2 + |x_j|^2 + 2 sum_k |x_ik x_jk|) (4x margin)."""
+    x = (xbits.astype(np.uint32) << 16).view(np.float32).astype(np.float64)
+    nrm = (x * x).sum(1)
+    ax = np.abs(x)
+    return 2.0 ** -20 * (nrm[:, None] + nrm[None, :] + 2 * ax @ ax.T)
+
+
+@pytest.mark.parametrize("n,d", [(1, 8), (5, 3), (128, 64), (300, 40), (1000, 128), (1029, 100), (2048, 64)])
+@pytest.mark.parametrize("kernel", ["gaussian", "dist2", "dist"])
+def test_pairmatrix_hd(tbs, n, d, kernel):
+    import torch
+    rng = np.random.default_rng(n * 131 + d)
+    xb = _bf16_bits(rng.random((n, d), dtype=np.float32))
+    xt = torch.from_numpy(xb.view(np.int16)).cuda().view(torch.bfloat16)
+    gamma = 1.0 / d
+    got = tbs.pairmatrix_hd(xt, gamma, kernel=kernel).cpu().numpy().astype(np.float64)
+    ref = oracle.pairmatrix_hd(xb, gamma, ktype=tbs.KERNELS[kernel])
+    B = _hd_bound(xb)
+    if kernel == "gaussian":
+        g32 = np.float64(np.float32(gamma))
+        tol = ref * (g32 * B + 2e-6) + 1e-30
+    elif kernel == "dist2":
+        tol = B + 1e-30
+    else:
+        tol = np.sqrt(B) + 1e-6 * ref
+    err = np.abs(got - ref)
+    assert np.all(err <= tol), (float(err.max()), float((err / tol).max()))
+
+
+def test_pairmatrix_hd_rows_and_host(tbs):
+    import torch
+    rng = np.random.default_rng(5)
+    xb = _bf16_bits(rng.standard_normal((700, 96)).astype(np.float32))
+    xt = torch.from_numpy(xb.view(np.int16)).cuda().view(torch.bfloat16)
+    full = tbs.pairmatrix_hd(xt, 0.01).cpu().numpy()
+    part = tbs.pairmatrix_hd(xt, 0.01, rows=(130, 419)).cpu().numpy()
+    assert np.array_equal(part, full[130:419])
+    host = np.empty((700, 700), np.float32)
+    assert tbs.lib().tbs_pairmatrix_hd(xb.ctypes.data, 700, 96, tbs._Kernel(0, 0.01), host.ctypes.data) == 0
+    assert np.array_equal(host, full)
+    ref = oracle.pairmatrix_hd(xb, 0.01)
+    assert np.all(np.abs(full - ref) <= ref * (0.01 * _hd_bound(xb) + 2e-6))

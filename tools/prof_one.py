@@ -23,6 +23,9 @@ elif wl == "pcf1m":
 elif wl == "sdh16k":
     p = torch.from_numpy(g.uniform(1 << 21, 4)).cuda()
     f = lambda: tbs.sdh(p, float(np.float32(math.sqrt(3) / 16384)), 16384)
+elif wl == "hd64k":
+    p = torch.from_numpy(g.uniform(1 << 16, 7, 64)).cuda().to(torch.bfloat16)
+    f = lambda: tbs.pairmatrix_hd(p, 1.0 / 64)
 elif wl == "pm64k":
     p = torch.from_numpy(g.uniform(1 << 16, 5)).cuda()
     f = lambda: tbs.pairmatrix(p, 1.0)
