@@ -1,4 +1,5 @@
 """Build libtbs.so (the C-ABI library) in-tree with nvcc for sm_100a."""
+import glob
 import os
 import subprocess
 import sys
@@ -7,8 +8,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libtbs.so")
 SRCS = [os.path.join(HERE, "csrc", f) for f in ("tbs_api.cu",)]
-DEPS = SRCS + [os.path.join(HERE, "csrc", f) for f in ("tbs_kernels.cuh", "tbs_ptx.cuh")] + \
-    [os.path.join(ROOT, "include", "tbs.h")]
+DEPS = SRCS + sorted(glob.glob(os.path.join(HERE, "csrc", "*.cuh"))) + [os.path.join(ROOT, "include", "tbs.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-shared", "-cudart", "static", "-Xptxas", "-v"]

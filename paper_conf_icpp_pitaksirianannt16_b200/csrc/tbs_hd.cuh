@@ -11,10 +11,11 @@
 //     64 bf16 of K per 16 KB box, completion on an mbarrier;
 //   * one thread issues tcgen05.mma.kind::f16 (M=128, N=128, K=16 steps, bf16 x bf16 -> fp32)
 //     into one of two TMEM accumulators (2 x 128 columns), tcgen05.commit -> mbarriers;
-//   * 8 epilogue warps tcgen05.ld the accumulator (32x32b.x32: warp w reads TMEM lanes
-//     32 (w % 4).. and columns 64 (w / 4)..), form s from the row / column norms, apply the
-//     kernel (ex2 for the Gaussian), stage the tile in shared memory, and write it with
-//     coalesced streaming 16-byte stores (each warp row = 512 contiguous bytes).
+//   * 16 epilogue warps tcgen05.ld the accumulator (32x32b.x32: warp w reads TMEM lanes
+//     32 (w % 4).. and columns 32 (w / 4)..), form s from the row / column norms (bulk-copied
+//     into shared memory by the producer beside the operands), apply the kernel (ex2 for the
+//     Gaussian), stage the tile in shared memory, and write it with coalesced streaming
+//     16-byte stores (each warp row = 512 contiguous bytes).
 // A dedicated producer warp overlaps the next tile's loads + MMAs with the epilogue.
 #pragma once
 #include <cstdint>
@@ -26,7 +27,7 @@ namespace hd {
 constexpr int kTile = 128;          // M = N = 128
 constexpr int kKBlock = 64;         // bf16 per 128-byte swizzle row (one TMA box = 128 x 64)
 constexpr int kMaxKBlocks = 2;      // d <= 128
-constexpr int kEpiWarps = 8;
+constexpr int kEpiWarps = 16;                    // 4 TMEM lane quarters x 4 column chunks of 32
 constexpr int kThreads = (kEpiWarps + 1) * 32;   // + one producer / MMA warp
 constexpr int kStageBytes = kTile * kKBlock * 2; // 16 KB
 constexpr int kStageRow = kTile + 4;             // staging row stride (floats): conflict-free
@@ -34,12 +35,13 @@ constexpr int kTmemCols = 256;                   // two 128-column fp32 accumula
 
 struct Smem {
   // offsets from the 1024-aligned dynamic smem base
-  static constexpr int A = 0;
-  static constexpr int B = A + kMaxKBlocks * kStageBytes;
-  static constexpr int STAGE = B + kMaxKBlocks * kStageBytes;
-  static constexpr int NORMS = STAGE + kTile * kStageRow * 4;
-  static constexpr int BARS = NORMS + kTile * 4;       // full, smem_free, acc_full[2], acc_empty[2]
-  static constexpr int TMEM = BARS + 6 * 8;
+  static constexpr int OPS = 0;                                  // [2 stages][A | B][kMaxKBlocks] x 16 KB
+  static constexpr int OPS_STAGE = 2 * kMaxKBlocks * kStageBytes;
+  static constexpr int STAGE = OPS + 2 * OPS_STAGE;              // output staging tile
+  static constexpr int NORMS = STAGE + kTile * kStageRow * 4;    // [4 slots][rows I | cols J] x 128 fp32
+  static constexpr int BARS = NORMS + 4 * 2 * kTile * 4;
+  // barriers: full[2] free[2] acc_full[2] acc_empty[2] nfull[4] nempty[4]
+  static constexpr int TMEM = BARS + 16 * 8;
   static constexpr int BYTES = TMEM + 16;
 };
 
@@ -69,6 +71,15 @@ __device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t a_desc, uint64_
       "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)
       : "memory");
 }
+// TMA 1-D bulk store shared -> global (bulk async-group completion), used to drain the
+// staged output tile without occupying the warps (SASS: UBLKCP).
+__device__ __forceinline__ void bulk_s2g(void* dst, uint32_t src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void named_bar(int id, int count) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
 }
@@ -123,23 +134,33 @@ __global__ void __launch_bounds__(kThreads, 1)
   extern __shared__ __align__(1024) unsigned char hd_smem_raw[];
   unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(hd_smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sbase = smem_addr(sm);
-  const uint32_t bar_full = sbase + Smem::BARS, bar_free = bar_full + 8;
-  const uint32_t bar_acc_full = bar_full + 16, bar_acc_empty = bar_full + 32;   // [2] each
+  const uint32_t b0 = sbase + Smem::BARS;
+  auto bar_full = [&](int s) { return b0 + 8 * s; };
+  auto bar_free = [&](int s) { return b0 + 16 + 8 * s; };
+  auto bar_acc_full = [&](int a) { return b0 + 32 + 8 * a; };
+  auto bar_acc_empty = [&](int a) { return b0 + 48 + 8 * a; };
+  auto bar_nfull = [&](int k) { return b0 + 64 + 8 * k; };
+  auto bar_nempty = [&](int k) { return b0 + 96 + 8 * k; };
   float* stage = reinterpret_cast<float*>(sm + Smem::STAGE);
-  float* snj = reinterpret_cast<float*>(sm + Smem::NORMS);
+  const float* snorm = reinterpret_cast<const float*>(sm + Smem::NORMS);        // [slot][2][128]
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(sm + Smem::TMEM);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int ntiles = tiles_i * tiles_j;
+  const long long ntiles = (long long)tiles_i * tiles_j;
+  // contiguous tile range per CTA (row-major: consecutive tiles share the row block I)
+  const long long t_beg = ntiles * blockIdx.x / gridDim.x, t_end = ntiles * (blockIdx.x + 1) / gridDim.x;
 
   if (warp == kEpiWarps) {
-    // producer warp: barriers + TMEM allocation (whole warp), then lane 0 drives TMA + MMA
     if (lane == 0) {
-      mbar_init(bar_full, 1);
-      mbar_init(bar_free, 1);
-      mbar_init(bar_acc_full, 1);
-      mbar_init(bar_acc_full + 8, 1);
-      mbar_init(bar_acc_empty, kEpiWarps);
-      mbar_init(bar_acc_empty + 8, kEpiWarps);
+      for (int k = 0; k < 2; ++k) {
+        mbar_init(bar_full(k), 1);
+        mbar_init(bar_free(k), 1);
+        mbar_init(bar_acc_full(k), 1);
+        mbar_init(bar_acc_empty(k), kEpiWarps);
+      }
+      for (int k = 0; k < 4; ++k) {
+        mbar_init(bar_nfull(k), 1);
+        mbar_init(bar_nempty(k), kEpiWarps);
+      }
       fence_mbar_init();
       asm volatile("prefetch.tensormap [%0];" ::"l"(&tmap) : "memory");
     }
@@ -156,86 +177,113 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   if (warp == kEpiWarps) {
     if (lane == 0) {
-      int it = 0;
-      for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++it) {
-        const int I = I0 + t / tiles_j, J = t % tiles_j, acc = it & 1;
-        if (it > 0) mbar_wait(bar_free, (uint32_t)((it - 1) & 1));          // previous MMAs done with smem
-        mbar_arrive_expect_tx(bar_full, (uint32_t)(2 * kblocks * kStageBytes));
+      // Producer / MMA issuer. Every wait below is on the completion right after the last
+      // one this thread consumed for that barrier, so no barrier can run two phases ahead.
+      auto issue = [&](int it, long long t) {
+        const int I = I0 + (int)(t / tiles_j), J = (int)(t % tiles_j), st = it & 1, ns = it & 3;
+        if (it >= 2) mbar_wait(bar_free(st), (uint32_t)(((it - 2) >> 1) & 1));     // MMAs of tile it-2 done
+        mbar_arrive_expect_tx(bar_full(st), (uint32_t)(2 * kblocks * kStageBytes));
+        const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
         for (int kb = 0; kb < kblocks; ++kb) {
-          tma_load_2d(sbase + Smem::A + kb * kStageBytes, &tmap, kb * kKBlock, I * kTile, bar_full);
-          tma_load_2d(sbase + Smem::B + kb * kStageBytes, &tmap, kb * kKBlock, J * kTile, bar_full);
+          tma_load_2d(ops + kb * kStageBytes, &tmap, kb * kKBlock, I * kTile, bar_full(st));
+          tma_load_2d(ops + (kMaxKBlocks + kb) * kStageBytes, &tmap, kb * kKBlock, J * kTile, bar_full(st));
         }
-        mbar_wait(bar_full, (uint32_t)(it & 1));
-        if (it >= 2) mbar_wait(bar_acc_empty + 8 * acc, (uint32_t)(((it - 2) >> 1) & 1));   // epilogue drained acc
+        if (it >= 4) mbar_wait(bar_nempty(ns), (uint32_t)(((it - 4) >> 2) & 1));   // epilogue of it-4 read slot
+        mbar_arrive_expect_tx(bar_nfull(ns), 2 * kTile * 4);
+        const uint32_t nd = sbase + Smem::NORMS + ns * 2 * kTile * 4;
+        bulk_g2s(nd, norms + I * kTile, kTile * 4, bar_nfull(ns));
+        bulk_g2s(nd + kTile * 4, norms + J * kTile, kTile * 4, bar_nfull(ns));
+      };
+      if (t_beg < t_end) issue(0, t_beg);
+      int it = 0;
+      for (long long t = t_beg; t < t_end; ++t, ++it) {
+        if (t + 1 < t_end) issue(it + 1, t + 1);                                    // run one tile ahead
+        const int st = it & 1, acc = it & 1;
+        mbar_wait(bar_full(st), (uint32_t)((it >> 1) & 1));
+        if (it >= 2) mbar_wait(bar_acc_empty(acc), (uint32_t)(((it - 2) >> 1) & 1));  // epilogue drained acc
         tc_fence_after();
         const uint32_t d_tmem = tmem + (uint32_t)(acc * kTile);
+        const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
         for (int kb = 0; kb < kblocks; ++kb) {
 #pragma unroll
           for (int ks = 0; ks < kKBlock / 16; ++ks) {
-            const uint64_t da = sw128_desc(sbase + Smem::A + kb * kStageBytes + ks * 32);
-            const uint64_t db = sw128_desc(sbase + Smem::B + kb * kStageBytes + ks * 32);
+            const uint64_t da = sw128_desc(ops + kb * kStageBytes + ks * 32);
+            const uint64_t db = sw128_desc(ops + (kMaxKBlocks + kb) * kStageBytes + ks * 32);
             tc_mma(d_tmem, da, db, kIdesc, (kb | ks) != 0 ? 1u : 0u);
           }
         }
-        tc_commit(bar_free);
-        tc_commit(bar_acc_full + 8 * acc);
+        tc_commit(bar_free(st));
+        tc_commit(bar_acc_full(acc));
       }
     }
   } else {
-    // epilogue warps: TMEM lane quarter q, column half h
-    const int q = warp & 3, h = warp >> 2;
-    const int et = threadIdx.x;        // 0..255
+    // epilogue warps: TMEM lane quarter q, 32-column chunk cq
+    const int q = warp & 3, cq = warp >> 2;
+    const int r = 32 * q + lane;
     int it = 0;
-    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++it) {
-      const int I = I0 + t / tiles_j, J = t % tiles_j, acc = it & 1;
-      named_bar(1, kEpiWarps * 32);                       // staging + column norms free
-      if (et < kTile) snj[et] = norms[J * kTile + et];
-      named_bar(1, kEpiWarps * 32);
-      const int r = 32 * q + lane;
-      const float ni = norms[I * kTile + r];
-      mbar_wait(bar_acc_full + 8 * acc, (uint32_t)((it >> 1) & 1));
+    for (long long t = t_beg; t < t_end; ++t, ++it) {
+      const int I = I0 + (int)(t / tiles_j), J = (int)(t % tiles_j), acc = it & 1, ns = it & 3;
+      const float* nrm = snorm + ns * 2 * kTile;
+      mbar_wait(bar_nfull(ns), (uint32_t)((it >> 2) & 1));
+      const float ni = nrm[r];
+      float nj[32];
+#pragma unroll
+      for (int x = 0; x < 32; ++x) nj[x] = nrm[kTile + 32 * cq + x];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(bar_nempty(ns));
+      mbar_wait(bar_acc_full(acc), (uint32_t)((it >> 1) & 1));
       tc_fence_after();
-#pragma unroll
-      for (int c = 0; c < 2; ++c) {
-        const int col0 = 64 * h + 32 * c;
-        uint32_t v[32];
-        tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + (uint32_t)(acc * kTile + col0), v);
-        float* srow = stage + r * kStageRow + col0;
-#pragma unroll
-        for (int x = 0; x < 32; x += 4) {
-          float o[4];
-#pragma unroll
-          for (int y = 0; y < 4; ++y) {
-            const float s = fmaf(-2.f, __uint_as_float(v[x + y]), ni + snj[col0 + x + y]);
-            if (KTYPE == 0) o[y] = ex2_approx(cexp * s);
-            else if (KTYPE == 1) o[y] = fmaxf(s, 0.f);
-            else o[y] = sqrt_approx(fmaxf(s, 0.f));
-          }
-          *reinterpret_cast<float4*>(srow + x) = make_float4(o[0], o[1], o[2], o[3]);
-        }
-      }
+      uint32_t v[32];
+      tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + (uint32_t)(acc * kTile + 32 * cq), v);
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(bar_acc_empty + 8 * acc);
+      if (lane == 0) mbar_arrive(bar_acc_empty(acc));
+      float o[32];
+#pragma unroll
+      for (int x = 0; x < 32; ++x) {
+        const float s = fmaf(-2.f, __uint_as_float(v[x]), ni + nj[x]);
+        if (KTYPE == 0) o[x] = ex2_approx(cexp * s);
+        else if (KTYPE == 1) o[x] = fmaxf(s, 0.f);
+        else o[x] = sqrt_approx(fmaxf(s, 0.f));
+      }
+      if (lane == 0) bulk_wait_read0();                   // this warp's bulk stores of the last tile read smem
+      named_bar(1, kEpiWarps * 32);                       // staging free
+      float* srow = stage + r * kStageRow + 32 * cq;
+#pragma unroll
+      for (int x = 0; x < 32; x += 4)
+        *reinterpret_cast<float4*>(srow + x) = make_float4(o[x], o[x + 1], o[x + 2], o[x + 3]);
+      fence_async_smem();                                 // generic-proxy writes -> visible to the TMA
       named_bar(1, kEpiWarps * 32);                       // tile staged
-      // coalesced streaming stores: warp w writes rows w, w+8, ... (512 B per row per warp)
-      const int jc = J * kTile + 4 * lane;
-      const bool vec = (n & 3) == 0 && jc + 3 < n;
-      for (int rr = warp; rr < kTile; rr += kEpiWarps) {
-        const int gi = I * kTile + rr;
-        if (gi < rb || gi >= re) continue;
-        float* dst = out + (size_t)(gi - rb) * (size_t)n + jc;
-        const float4 val = *reinterpret_cast<const float4*>(stage + rr * kStageRow + 4 * lane);
-        if (vec) {
-          st_cs_v4(dst, val.x, val.y, val.z, val.w);
-        } else {
-          if (jc < n) __stcs(dst, val.x);
-          if (jc + 1 < n) __stcs(dst + 1, val.y);
-          if (jc + 2 < n) __stcs(dst + 2, val.z);
-          if (jc + 3 < n) __stcs(dst + 3, val.w);
+      const int j0 = J * kTile;
+      if ((n & 3) == 0 && j0 + kTile <= n) {
+        // full-width tile: lane l of warp w bulk-stores row w + 16 k for k = l (8 rows / warp)
+        if (lane < kTile / kEpiWarps) {
+          const int rr = warp + kEpiWarps * lane;
+          const int gi = I * kTile + rr;
+          if (gi >= rb && gi < re)
+            bulk_s2g(out + (size_t)(gi - rb) * (size_t)n + j0, smem_addr(stage + rr * kStageRow), kTile * 4);
+          bulk_commit();
+        }
+      } else {
+        // ragged right edge: coalesced streaming stores, masked
+        const int jc = j0 + 4 * lane;
+        for (int rr = warp; rr < kTile; rr += kEpiWarps) {
+          const int gi = I * kTile + rr;
+          const float4 val = *reinterpret_cast<const float4*>(stage + rr * kStageRow + 4 * lane);
+          if (gi < rb || gi >= re) continue;
+          float* dst = out + (size_t)(gi - rb) * (size_t)n + jc;
+          if ((n & 3) == 0 && jc + 3 < n) {
+            st_cs_v4(dst, val.x, val.y, val.z, val.w);
+          } else {
+            if (jc < n) __stcs(dst, val.x);
+            if (jc + 1 < n) __stcs(dst + 1, val.y);
+            if (jc + 2 < n) __stcs(dst + 2, val.z);
+            if (jc + 3 < n) __stcs(dst + 3, val.w);
+          }
         }
       }
     }
+    if (lane < kTile / kEpiWarps) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // writes done
   }
   tc_fence_before();
   __syncthreads();
