@@ -593,7 +593,8 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
   }
   EncodeTiledFn enc = nullptr;
   if (!rc) rc = encode_tiled_fn(enc);
-  CUtensorMap tmap;
+  CUtensorMap tmap, tmap_out;
+  const int use_tma_store = (n % 4) == 0;
   if (!rc) {
     const cuuint64_t dims[2] = {(cuuint64_t)dp, (cuuint64_t)n_pad};
     const cuuint64_t strides[1] = {(cuuint64_t)dp * 2};
@@ -603,6 +604,21 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
                             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (cr != CUDA_SUCCESS) rc = fail(TBS_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)cr);
+  }
+  if (!rc) {
+    // output rows [rb, re) x n fp32; TMA boxes of 128 rows x 32 columns, 128-byte swizzle
+    const cuuint64_t dims[2] = {(cuuint64_t)n, (cuuint64_t)(re - rb)};
+    const cuuint64_t strides[1] = {(cuuint64_t)n * 4};
+    const cuuint32_t box[2] = {(cuuint32_t)hd::kBoxCols, (cuuint32_t)hd::kTile};
+    const cuuint32_t estr[2] = {1, 1};
+    if (use_tma_store) {
+      const CUresult cr = enc(&tmap_out, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, out, dims, strides, box, estr,
+                              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                              CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      if (cr != CUDA_SUCCESS) rc = fail(TBS_ECUDA, "cuTensorMapEncodeTiled (output) failed (%d)", (int)cr);
+    } else {
+      memset(&tmap_out, 0, sizeof(tmap_out));
+    }
   }
   if (!rc) {
     const int I0 = (int)(rb / hd::kTile), I1 = (int)((re + hd::kTile - 1) / hd::kTile);
@@ -615,8 +631,8 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
     auto launch = [&](auto kern) -> int {
       TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
       if (eb) TBS_CUDA(cudaEventRecord(eb, st));
-      kern<<<grid, hd::kThreads, smem, st>>>(tmap, norms, (int)n, kblocks, I0, tiles_i, tiles_j, (int)rb, (int)re,
-                                             cexp, out);
+      kern<<<grid, hd::kThreads, smem, st>>>(tmap, tmap_out, use_tma_store, norms, (int)n, kblocks, I0, tiles_i,
+                                             tiles_j, (int)rb, (int)re, cexp, out);
       TBS_CUDA(cudaGetLastError());
       g_launches.fetch_add(1);
       if (ee) TBS_CUDA(cudaEventRecord(ee, st));

@@ -30,7 +30,7 @@ constexpr int kMaxKBlocks = 2;      // d <= 128
 constexpr int kEpiWarps = 16;                    // 4 TMEM lane quarters x 4 column chunks of 32
 constexpr int kThreads = (kEpiWarps + 1) * 32;   // + one producer / MMA warp
 constexpr int kStageBytes = kTile * kKBlock * 2; // 16 KB
-constexpr int kStageRow = kTile + 4;             // staging row stride (floats): conflict-free
+constexpr int kBoxCols = 32;                     // output TMA box: 128 rows x 32 fp32 (128 B, SWIZZLE_128B)
 constexpr int kTmemCols = 256;                   // two 128-column fp32 accumulators
 
 struct Smem {
@@ -38,7 +38,7 @@ struct Smem {
   static constexpr int OPS = 0;                                  // [2 stages][A | B][kMaxKBlocks] x 16 KB
   static constexpr int OPS_STAGE = 2 * kMaxKBlocks * kStageBytes;
   static constexpr int STAGE = OPS + 2 * OPS_STAGE;              // output staging tile
-  static constexpr int NORMS = STAGE + kTile * kStageRow * 4;    // [4 slots][rows I | cols J] x 128 fp32
+  static constexpr int NORMS = STAGE + kTile * kTile * 4;        // [4 slots][rows I | cols J] x 128 fp32
   static constexpr int BARS = NORMS + 4 * 2 * kTile * 4;
   // barriers: full[2] free[2] acc_full[2] acc_empty[2] nfull[4] nempty[4]
   static constexpr int TMEM = BARS + 16 * 8;
@@ -80,6 +80,46 @@ __device__ __forceinline__ void bulk_s2g(void* dst, uint32_t src, uint32_t bytes
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+// 2-D TMA tensor store shared -> global with an L2 eviction-priority hint.
+__device__ __forceinline__ void tma_store_2d(const void* tmap, int c0, int c1, uint32_t src, uint64_t policy) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%1, %2}], [%3], %4;" ::"l"(
+                   tmap),
+               "r"(c0), "r"(c1), "r"(src), "l"(policy)
+               : "memory");
+}
+__device__ __forceinline__ void tma_load_2d_hint(uint32_t dst, const void* tmap, int c0, int c1, uint32_t bar,
+                                                 uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%2, %3}], "
+      "[%4], %5;" ::"r"(dst),
+      "l"(tmap), "r"(c0), "r"(c1), "r"(bar), "l"(policy)
+      : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void st_shared_v4(uint32_t a, float x, float y, float z, float w) {
+  asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a), "f"(x), "f"(y), "f"(z), "f"(w) : "memory");
+}
+__device__ __forceinline__ float ld_shared_f32(uint32_t a) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a) : "memory");
+  return v;
+}
+// Byte offset of output element (row, col) in the staging tile: 4 boxes of 128 rows x 32 fp32
+// (one per 32-column chunk), each row 128 B with the TMA SWIZZLE_128B pattern (16-byte chunk
+// index XOR row % 8) — conflict-free for one-row-per-lane writes, and the layout a 2-D TMA
+// store of a [128 x 32] box with SWIZZLE_128B reads.
+__device__ __forceinline__ uint32_t stage_off(int row, int col) {
+  return (uint32_t)((col >> 5) * (kTile * 128) + row * 128 + ((((col & 31) >> 2) ^ (row & 7)) << 4) + (col & 3) * 4);
+}
 __device__ __forceinline__ void named_bar(int id, int count) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
 }
@@ -129,8 +169,9 @@ __global__ void hd_prep(const uint16_t* __restrict__ x, int n, int d, int n_pad,
 
 template <int KTYPE>
 __global__ void __launch_bounds__(kThreads, 1)
-    hd_pairmatrix_kernel(const __grid_constant__ CUtensorMap tmap, const float* __restrict__ norms, int n, int kblocks,
-                         int I0, int tiles_i, int tiles_j, int rb, int re, float cexp, float* __restrict__ out) {
+    hd_pairmatrix_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ CUtensorMap tmap_out,
+                         int use_tma_store, const float* __restrict__ norms, int n, int kblocks, int I0, int tiles_i,
+                         int tiles_j, int rb, int re, float cexp, float* __restrict__ out) {
   extern __shared__ __align__(1024) unsigned char hd_smem_raw[];
   unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(hd_smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sbase = smem_addr(sm);
@@ -141,8 +182,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   auto bar_acc_empty = [&](int a) { return b0 + 48 + 8 * a; };
   auto bar_nfull = [&](int k) { return b0 + 64 + 8 * k; };
   auto bar_nempty = [&](int k) { return b0 + 96 + 8 * k; };
-  float* stage = reinterpret_cast<float*>(sm + Smem::STAGE);
-  const float* snorm = reinterpret_cast<const float*>(sm + Smem::NORMS);        // [slot][2][128]
+  const uint32_t stage = sbase + Smem::STAGE;
+  const uint32_t snorm = sbase + Smem::NORMS;                                   // [slot][2][128] fp32
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(sm + Smem::TMEM);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const long long ntiles = (long long)tiles_i * tiles_j;
@@ -163,6 +204,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       fence_mbar_init();
       asm volatile("prefetch.tensormap [%0];" ::"l"(&tmap) : "memory");
+      asm volatile("prefetch.tensormap [%0];" ::"l"(&tmap_out) : "memory");
     }
     __syncwarp();
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_addr(tmem_holder)),
@@ -179,14 +221,15 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (lane == 0) {
       // Producer / MMA issuer. Every wait below is on the completion right after the last
       // one this thread consumed for that barrier, so no barrier can run two phases ahead.
+      const uint64_t keep = policy_evict_last();
       auto issue = [&](int it, long long t) {
         const int I = I0 + (int)(t / tiles_j), J = (int)(t % tiles_j), st = it & 1, ns = it & 3;
         if (it >= 2) mbar_wait(bar_free(st), (uint32_t)(((it - 2) >> 1) & 1));     // MMAs of tile it-2 done
         mbar_arrive_expect_tx(bar_full(st), (uint32_t)(2 * kblocks * kStageBytes));
         const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
-        for (int kb = 0; kb < kblocks; ++kb) {
-          tma_load_2d(ops + kb * kStageBytes, &tmap, kb * kKBlock, I * kTile, bar_full(st));
-          tma_load_2d(ops + (kMaxKBlocks + kb) * kStageBytes, &tmap, kb * kKBlock, J * kTile, bar_full(st));
+        for (int kb = 0; kb < kblocks; ++kb) {   // features stay L2-resident (evict_last) under the output stream
+          tma_load_2d_hint(ops + kb * kStageBytes, &tmap, kb * kKBlock, I * kTile, bar_full(st), keep);
+          tma_load_2d_hint(ops + (kMaxKBlocks + kb) * kStageBytes, &tmap, kb * kKBlock, J * kTile, bar_full(st), keep);
         }
         if (it >= 4) mbar_wait(bar_nempty(ns), (uint32_t)(((it - 4) >> 2) & 1));   // epilogue of it-4 read slot
         mbar_arrive_expect_tx(bar_nfull(ns), 2 * kTile * 4);
@@ -220,15 +263,17 @@ __global__ void __launch_bounds__(kThreads, 1)
     // epilogue warps: TMEM lane quarter q, 32-column chunk cq
     const int q = warp & 3, cq = warp >> 2;
     const int r = 32 * q + lane;
+    const uint64_t stream_out = policy_evict_first();
+    const bool storer = threadIdx.x == 0;                 // issues the tile's four TMA stores
     int it = 0;
     for (long long t = t_beg; t < t_end; ++t, ++it) {
       const int I = I0 + (int)(t / tiles_j), J = (int)(t % tiles_j), acc = it & 1, ns = it & 3;
-      const float* nrm = snorm + ns * 2 * kTile;
+      const uint32_t nrm = snorm + ns * 2 * kTile * 4;
       mbar_wait(bar_nfull(ns), (uint32_t)((it >> 2) & 1));
-      const float ni = nrm[r];
+      const float ni = ld_shared_f32(nrm + 4 * r);
       float nj[32];
 #pragma unroll
-      for (int x = 0; x < 32; ++x) nj[x] = nrm[kTile + 32 * cq + x];
+      for (int x = 0; x < 32; ++x) nj[x] = ld_shared_f32(nrm + 4 * (kTile + 32 * cq + x));
       __syncwarp();
       if (lane == 0) mbar_arrive(bar_nempty(ns));
       mbar_wait(bar_acc_full(acc), (uint32_t)((it >> 1) & 1));
@@ -246,44 +291,36 @@ __global__ void __launch_bounds__(kThreads, 1)
         else if (KTYPE == 1) o[x] = fmaxf(s, 0.f);
         else o[x] = sqrt_approx(fmaxf(s, 0.f));
       }
-      if (lane == 0) bulk_wait_read0();                   // this warp's bulk stores of the last tile read smem
+      if (storer) bulk_wait_read0();                      // last tile's TMA stores have read the staging
       named_bar(1, kEpiWarps * 32);                       // staging free
-      float* srow = stage + r * kStageRow + 32 * cq;
 #pragma unroll
       for (int x = 0; x < 32; x += 4)
-        *reinterpret_cast<float4*>(srow + x) = make_float4(o[x], o[x + 1], o[x + 2], o[x + 3]);
+        st_shared_v4(stage + stage_off(r, 32 * cq + x), o[x], o[x + 1], o[x + 2], o[x + 3]);
       fence_async_smem();                                 // generic-proxy writes -> visible to the TMA
       named_bar(1, kEpiWarps * 32);                       // tile staged
-      const int j0 = J * kTile;
-      if ((n & 3) == 0 && j0 + kTile <= n) {
-        // full-width tile: lane l of warp w bulk-stores row w + 16 k for k = l (8 rows / warp)
-        if (lane < kTile / kEpiWarps) {
-          const int rr = warp + kEpiWarps * lane;
-          const int gi = I * kTile + rr;
-          if (gi >= rb && gi < re)
-            bulk_s2g(out + (size_t)(gi - rb) * (size_t)n + j0, smem_addr(stage + rr * kStageRow), kTile * 4);
+      if (use_tma_store && I * kTile >= rb) {
+        // TMA clips the box past the last row / column (ragged edges); a tile starting above
+        // the row range (negative box origin) takes the masked path below
+        if (storer) {
+#pragma unroll
+          for (int c = 0; c < kTile / kBoxCols; ++c)
+            tma_store_2d(&tmap_out, J * kTile + c * kBoxCols, I * kTile - rb, stage + c * kTile * 128, stream_out);
           bulk_commit();
         }
       } else {
-        // ragged right edge: coalesced streaming stores, masked
-        const int jc = j0 + 4 * lane;
+        // n % 4 != 0 (row pitch not 16-byte aligned) or first partial tile row: masked stores
+        const int jc = J * kTile + lane;
         for (int rr = warp; rr < kTile; rr += kEpiWarps) {
           const int gi = I * kTile + rr;
-          const float4 val = *reinterpret_cast<const float4*>(stage + rr * kStageRow + 4 * lane);
           if (gi < rb || gi >= re) continue;
-          float* dst = out + (size_t)(gi - rb) * (size_t)n + jc;
-          if ((n & 3) == 0 && jc + 3 < n) {
-            st_cs_v4(dst, val.x, val.y, val.z, val.w);
-          } else {
-            if (jc < n) __stcs(dst, val.x);
-            if (jc + 1 < n) __stcs(dst + 1, val.y);
-            if (jc + 2 < n) __stcs(dst + 2, val.z);
-            if (jc + 3 < n) __stcs(dst + 3, val.w);
-          }
+          float* dst = out + (size_t)(gi - rb) * (size_t)n;
+#pragma unroll
+          for (int cc = 0; cc < kTile; cc += 32)
+            if (jc + cc < n) __stcs(dst + jc + cc, ld_shared_f32(stage + stage_off(rr, lane + cc)));
         }
       }
     }
-    if (lane < kTile / kEpiWarps) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // writes done
+    if (storer) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // all TMA stores complete
   }
   tc_fence_before();
   __syncthreads();
