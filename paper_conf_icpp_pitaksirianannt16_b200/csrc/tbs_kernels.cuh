@@ -28,7 +28,7 @@ namespace tbs {
 constexpr int kThreads = 256;              // 8 warps per CTA
 constexpr int kPUnroll = TBS_PUNROLL;
 constexpr int kWarps = kThreads / 32;
-constexpr int kPadAlign = 2048;            // SoA rows padded to a multiple of every anchor tile / chunk
+constexpr int kPadAlign = 4096;            // SoA rows padded to a multiple of every anchor tile / chunk
 constexpr uint32_t kMagic = 0x4B000000u;   // bits of 2^23: x + 2^23 (round-down) = 2^23 + floor(x)
 constexpr float kMagicF = 8388608.0f;
 constexpr int kNoAnchor = 0x7fffffff;      // masked anchor index (no partner is greater)
