@@ -47,6 +47,7 @@ WORKLOADS = {
     "pairmatrix_64k": ("pairmatrix", "uniform", 1 << 16, 5, dict(gamma=1.0)),  # configs[4]
     "kde_uniform_1m": ("kde", "uniform", 1 << 20, 2, dict(gamma=1.0)),        # NEXT-2 (Type-I float sum)
     "pairmatrix_hd_64k_d64": ("pairmatrix_hd", "uniform", 1 << 16, 7, dict(d=64, gamma=1.0 / 64)),  # NEXT-3
+    "pairmatrix_hd_64k_d512": ("pairmatrix_hd", "uniform", 1 << 16, 7, dict(d=512, gamma=1.0 / 512)),
 }
 METRIC = "SDH pair-distances/sec (G pairs/s) at N=1M–4M, 1/2/4/8 B200, % of roofline"
 
@@ -70,6 +71,8 @@ def peaks():
         atoms=SMS * ATOMS_LANES_PER_CLK_SM * f_max,
         mufu=SMS * MUFU_LANES_PER_CLK_SM * f_max,
         hbm=float(mp.get("hbm_gbs", 6650.0)) * 1e9,
+        bf16=float(mp.get("bf16_tflops", 2250.0)) * 1e12,
+        bf16_src="MEASURED_PEAKS.json bf16_tflops" if "bf16_tflops" in mp else "fallback 2.25 PF nominal",
         hbm_src="MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in mp else "fallback 6.65 TB/s (B200_PROFILING.md)",
     )
 
@@ -310,6 +313,20 @@ def main():
         roof = {"bound": "hbm", "achieved": achieved / 1e9, "peak": pk["hbm"] / 1e9, "unit": "GB/s",
                 "frac": achieved / pk["hbm"], "peak_source": pk["hbm_src"],
                 "algorithmic_bytes_per_launch": bytes_}
+        if op == "pairmatrix_hd":
+            # the Gram contraction: 2 d flops per entry on the bf16 tensor cores; the bound is
+            # whichever of (output bytes / HBM, flops / tensor peak) takes longer
+            flops = 2.0 * params["d"] * rank_units
+            tfrac = flops / (kavg * 1e-3) / pk["bf16"]
+            roof["tensor_view"] = {"achieved": flops / (kavg * 1e-3) / 1e12, "peak": pk["bf16"] / 1e12,
+                                   "unit": "TFLOP/s", "frac": tfrac, "peak_source": pk["bf16_src"],
+                                   "algorithmic_flops_per_launch": flops}
+            if flops / pk["bf16"] > bytes_ / pk["hbm"]:
+                roof = {"bound": "tensor", "achieved": flops / (kavg * 1e-3) / 1e12, "peak": pk["bf16"] / 1e12,
+                        "unit": "TFLOP/s", "frac": tfrac, "peak_source": pk["bf16_src"],
+                        "algorithmic_flops_per_launch": flops,
+                        "hbm_view": {"achieved": achieved / 1e9, "peak": pk["hbm"] / 1e9, "unit": "GB/s",
+                                     "frac": achieved / pk["hbm"]}}
     else:
         rb, re = tbs.rank_rows(n, world, rank)
         rank_units = (re - rb) * (2 * n - rb - re - 1) // 2

@@ -127,7 +127,7 @@ int tbs_rdf(const uint64_t* hist, int nbuckets, int dim, float bucket_width, int
 
 /* High-dimensional Type-III pair matrix on the 5th-generation tensor cores (NEXT-3;
  * PAPER.md L330-332 kernel methods over feature spaces): features are bf16 [n][d] row-major
- * (raw 16-bit patterns), 1 <= d <= 128 (larger d: TBS_EUNSUPPORTED). out[i*n + j] = K(x_i, x_j)
+ * (raw 16-bit patterns), 1 <= d <= 1024 (larger d: TBS_EUNSUPPORTED). out[i*n + j] = K(x_i, x_j)
  * in fp32 for all i, j (diagonal included) with s = |x_i|^2 + |x_j|^2 - 2 x_i.x_j from
  * tcgen05 bf16 x bf16 -> fp32 dot products (error ~2^-22 (|x_i|^2 + |x_j|^2) on s), clamped
  * at 0 for the distance kernels. Host or device pointers, synchronous. */

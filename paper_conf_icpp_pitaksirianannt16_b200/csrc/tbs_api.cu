@@ -568,7 +568,7 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
             cudaEvent_t eb, cudaEvent_t ee) {
   if (n < 0 || n > (1 << 24)) return fail(TBS_EINVAL, "n out of range for the pair matrix");
   if (d < 1) return fail(TBS_EINVAL, "d must be >= 1");
-  if (d > hd::kKBlock * hd::kMaxKBlocks) return fail(TBS_EUNSUPPORTED, "d > 128 not supported yet");
+  if (d > hd::kMaxD) return fail(TBS_EUNSUPPORTED, "d > %d not supported", hd::kMaxD);
   if (rb < 0 || re < rb || re > n) return fail(TBS_EINVAL, "row range outside [0, n]");
   if (k.type < 0 || k.type > 2) return fail(TBS_EINVAL, "kernel type %d unknown", k.type);
   if (k.type == TBS_K_GAUSSIAN && !std::isfinite(k.gamma)) return fail(TBS_EINVAL, "gamma must be finite");
@@ -577,7 +577,7 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
   Device dev;
   int rc = current_device(dev);
   if (rc) return rc;
-  const int dp = d <= hd::kKBlock ? hd::kKBlock : 2 * hd::kKBlock;
+  const int dp = (d + hd::kKBlock - 1) / hd::kKBlock * hd::kKBlock;
   const int64_t n_pad = (n + hd::kTile - 1) / hd::kTile * hd::kTile;
   unsigned char* scratch = nullptr;
   const size_t xbytes = (size_t)n_pad * dp * 2;

@@ -26,7 +26,8 @@ namespace hd {
 
 constexpr int kTile = 128;          // M = N = 128
 constexpr int kKBlock = 64;         // bf16 per 128-byte swizzle row (one TMA box = 128 x 64)
-constexpr int kMaxKBlocks = 2;      // d <= 128
+constexpr int kRing = 4;            // operand ring: 4 stages of (A, B) k-blocks = 128 KB
+constexpr int kMaxD = 1024;         // feature dimension limit (k-blocks stream through the ring)
 constexpr int kEpiWarps = 16;                    // 4 TMEM lane quarters x 4 column chunks of 32
 constexpr int kThreads = (kEpiWarps + 1) * 32;   // + one producer / MMA warp
 constexpr int kStageBytes = kTile * kKBlock * 2; // 16 KB
@@ -35,13 +36,13 @@ constexpr int kTmemCols = 256;                   // two 128-column fp32 accumula
 
 struct Smem {
   // offsets from the 1024-aligned dynamic smem base
-  static constexpr int OPS = 0;                                  // [2 stages][A | B][kMaxKBlocks] x 16 KB
-  static constexpr int OPS_STAGE = 2 * kMaxKBlocks * kStageBytes;
-  static constexpr int STAGE = OPS + 2 * OPS_STAGE;              // output staging tile
+  static constexpr int OPS = 0;                                  // [kRing][A | B] x 16 KB
+  static constexpr int OPS_STAGE = 2 * kStageBytes;
+  static constexpr int STAGE = OPS + kRing * OPS_STAGE;          // output staging tile (4 swizzled boxes)
   static constexpr int NORMS = STAGE + kTile * kTile * 4;        // [4 slots][rows I | cols J] x 128 fp32
   static constexpr int BARS = NORMS + 4 * 2 * kTile * 4;
-  // barriers: full[2] free[2] acc_full[2] acc_empty[2] nfull[4] nempty[4]
-  static constexpr int TMEM = BARS + 16 * 8;
+  // barriers: full[kRing] free[kRing] acc_full[2] acc_empty[2] nfull[4] nempty[4]
+  static constexpr int TMEM = BARS + (2 * kRing + 12) * 8;
   static constexpr int BYTES = TMEM + 16;
 };
 
@@ -177,11 +178,11 @@ __global__ void __launch_bounds__(kThreads, 1)
   const uint32_t sbase = smem_addr(sm);
   const uint32_t b0 = sbase + Smem::BARS;
   auto bar_full = [&](int s) { return b0 + 8 * s; };
-  auto bar_free = [&](int s) { return b0 + 16 + 8 * s; };
-  auto bar_acc_full = [&](int a) { return b0 + 32 + 8 * a; };
-  auto bar_acc_empty = [&](int a) { return b0 + 48 + 8 * a; };
-  auto bar_nfull = [&](int k) { return b0 + 64 + 8 * k; };
-  auto bar_nempty = [&](int k) { return b0 + 96 + 8 * k; };
+  auto bar_free = [&](int s) { return b0 + 8 * (kRing + s); };
+  auto bar_acc_full = [&](int a) { return b0 + 8 * (2 * kRing + a); };
+  auto bar_acc_empty = [&](int a) { return b0 + 8 * (2 * kRing + 2 + a); };
+  auto bar_nfull = [&](int k) { return b0 + 8 * (2 * kRing + 4 + k); };
+  auto bar_nempty = [&](int k) { return b0 + 8 * (2 * kRing + 8 + k); };
   const uint32_t stage = sbase + Smem::STAGE;
   const uint32_t snorm = sbase + Smem::NORMS;                                   // [slot][2][128] fp32
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(sm + Smem::TMEM);
@@ -192,9 +193,11 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   if (warp == kEpiWarps) {
     if (lane == 0) {
-      for (int k = 0; k < 2; ++k) {
+      for (int k = 0; k < kRing; ++k) {
         mbar_init(bar_full(k), 1);
         mbar_init(bar_free(k), 1);
+      }
+      for (int k = 0; k < 2; ++k) {
         mbar_init(bar_acc_full(k), 1);
         mbar_init(bar_acc_empty(k), kEpiWarps);
       }
@@ -222,40 +225,51 @@ __global__ void __launch_bounds__(kThreads, 1)
       // Producer / MMA issuer. Every wait below is on the completion right after the last
       // one this thread consumed for that barrier, so no barrier can run two phases ahead.
       const uint64_t keep = policy_evict_last();
-      auto issue = [&](int it, long long t) {
-        const int I = I0 + (int)(t / tiles_j), J = (int)(t % tiles_j), st = it & 1, ns = it & 3;
-        if (it >= 2) mbar_wait(bar_free(st), (uint32_t)(((it - 2) >> 1) & 1));     // MMAs of tile it-2 done
-        mbar_arrive_expect_tx(bar_full(st), (uint32_t)(2 * kblocks * kStageBytes));
-        const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
-        for (int kb = 0; kb < kblocks; ++kb) {   // features stay L2-resident (evict_last) under the output stream
-          tma_load_2d_hint(ops + kb * kStageBytes, &tmap, kb * kKBlock, I * kTile, bar_full(st), keep);
-          tma_load_2d_hint(ops + (kMaxKBlocks + kb) * kStageBytes, &tmap, kb * kKBlock, J * kTile, bar_full(st), keep);
+      // Operand k-blocks of consecutive tiles stream through a kRing-deep ring; loads run up
+      // to kRing k-blocks ahead of the MMAs. A tile's norms go into a 4-slot ring with its
+      // first k-block.
+      const long long total = (t_end - t_beg) * (long long)kblocks;
+      long long gl = 0;                                   // next k-block to load
+      auto load_next = [&]() {
+        const int st = (int)(gl % kRing);
+        if (gl >= kRing) mbar_wait(bar_free(st), (uint32_t)(((gl / kRing) - 1) & 1));   // MMAs of gl-kRing done
+        const long long ti = gl / kblocks;
+        const int kb = (int)(gl % kblocks);
+        const long long t = t_beg + ti;
+        const int I = I0 + (int)(t / tiles_j), J = (int)(t % tiles_j);
+        if (kb == 0) {
+          const int ns = (int)(ti & 3);
+          if (ti >= 4) mbar_wait(bar_nempty(ns), (uint32_t)(((ti - 4) >> 2) & 1));      // epilogue of ti-4 read slot
+          mbar_arrive_expect_tx(bar_nfull(ns), 2 * kTile * 4);
+          const uint32_t nd = sbase + Smem::NORMS + ns * 2 * kTile * 4;
+          bulk_g2s(nd, norms + I * kTile, kTile * 4, bar_nfull(ns));
+          bulk_g2s(nd + kTile * 4, norms + J * kTile, kTile * 4, bar_nfull(ns));
         }
-        if (it >= 4) mbar_wait(bar_nempty(ns), (uint32_t)(((it - 4) >> 2) & 1));   // epilogue of it-4 read slot
-        mbar_arrive_expect_tx(bar_nfull(ns), 2 * kTile * 4);
-        const uint32_t nd = sbase + Smem::NORMS + ns * 2 * kTile * 4;
-        bulk_g2s(nd, norms + I * kTile, kTile * 4, bar_nfull(ns));
-        bulk_g2s(nd + kTile * 4, norms + J * kTile, kTile * 4, bar_nfull(ns));
+        mbar_arrive_expect_tx(bar_full(st), (uint32_t)(2 * kStageBytes));
+        const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
+        // features stay L2-resident (evict_last) under the output stream
+        tma_load_2d_hint(ops, &tmap, kb * kKBlock, I * kTile, bar_full(st), keep);
+        tma_load_2d_hint(ops + kStageBytes, &tmap, kb * kKBlock, J * kTile, bar_full(st), keep);
+        ++gl;
       };
-      if (t_beg < t_end) issue(0, t_beg);
       int it = 0;
       for (long long t = t_beg; t < t_end; ++t, ++it) {
-        if (t + 1 < t_end) issue(it + 1, t + 1);                                    // run one tile ahead
-        const int st = it & 1, acc = it & 1;
-        mbar_wait(bar_full(st), (uint32_t)((it >> 1) & 1));
-        if (it >= 2) mbar_wait(bar_acc_empty(acc), (uint32_t)(((it - 2) >> 1) & 1));  // epilogue drained acc
-        tc_fence_after();
+        const int acc = it & 1;
         const uint32_t d_tmem = tmem + (uint32_t)(acc * kTile);
-        const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
         for (int kb = 0; kb < kblocks; ++kb) {
+          const long long gm = (long long)it * kblocks + kb;   // k-block consumed now
+          while (gl < total && gl < gm + kRing) load_next();
+          const int st = (int)(gm % kRing);
+          mbar_wait(bar_full(st), (uint32_t)((gm / kRing) & 1));
+          if (kb == 0 && it >= 2) mbar_wait(bar_acc_empty(acc), (uint32_t)(((it - 2) >> 1) & 1));  // acc drained
+          tc_fence_after();
+          const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
 #pragma unroll
-          for (int ks = 0; ks < kKBlock / 16; ++ks) {
-            const uint64_t da = sw128_desc(ops + kb * kStageBytes + ks * 32);
-            const uint64_t db = sw128_desc(ops + (kMaxKBlocks + kb) * kStageBytes + ks * 32);
-            tc_mma(d_tmem, da, db, kIdesc, (kb | ks) != 0 ? 1u : 0u);
-          }
+          for (int ks = 0; ks < kKBlock / 16; ++ks)
+            tc_mma(d_tmem, sw128_desc(ops + ks * 32), sw128_desc(ops + kStageBytes + ks * 32), kIdesc,
+                   (kb | ks) != 0 ? 1u : 0u);
+          tc_commit(bar_free(st));
         }
-        tc_commit(bar_free(st));
         tc_commit(bar_acc_full(acc));
       }
     }

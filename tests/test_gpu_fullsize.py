@@ -185,5 +185,5 @@ def test_pairmatrix_hd_64k_sampled_rows(tbs):
     g32 = np.float64(np.float32(1.0 / d))
     for k, r in enumerate(rows):
         ref = oracle.pairmatrix_hd(xb, 1.0 / d, rows=(r, r + 1))[0]
-        B = 2.0 ** -20 * (nrm[r] + nrm + 2 * np.abs(xf) @ np.abs(xf[r]))
+        B = 2.0 ** -23 * (d / 16 + 8) * (nrm[r] + nrm + 2 * np.abs(xf) @ np.abs(xf[r]))
         assert np.all(np.abs(got[k] - ref) <= ref * (g32 * B + 2e-6)), r

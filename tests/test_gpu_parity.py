@@ -342,15 +342,17 @@ def _bf16_bits(a):
 
 
 def _hd_bound(xbits):
-    """Per-entry bound on |s_gpu - s|: fp32 norms and fp32 tensor-core accumulation
-    of exact bf16 products, 2^-20 (|x_i|^2 + |x_j|^2 + 2 sum_k |x_ik x_jk|) (4x margin)."""
+    """Per-entry bound on |s_gpu - s|: exact bf16 products, fp32 accumulation in
+    the tensor core (K-chunks of 16 summed in sequence) and in the norms:
+    2^-23 (d/16 + 8) (|x_i|^2 + |x_j|^2 + 2 sum_k |x_ik x_jk|)."""
     x = (xbits.astype(np.uint32) << 16).view(np.float32).astype(np.float64)
     nrm = (x * x).sum(1)
     ax = np.abs(x)
-    return 2.0 ** -20 * (nrm[:, None] + nrm[None, :] + 2 * ax @ ax.T)
+    return 2.0 ** -23 * (x.shape[1] / 16 + 8) * (nrm[:, None] + nrm[None, :] + 2 * ax @ ax.T)
 
 
-@pytest.mark.parametrize("n,d", [(1, 8), (5, 3), (128, 64), (300, 40), (1000, 128), (1029, 100), (2048, 64)])
+@pytest.mark.parametrize("n,d", [(1, 8), (5, 3), (128, 64), (300, 40), (1000, 128), (1029, 100), (2048, 64),
+                                 (777, 192), (520, 256), (300, 512), (257, 1000)])
 @pytest.mark.parametrize("kernel", ["gaussian", "dist2", "dist"])
 def test_pairmatrix_hd(tbs, n, d, kernel):
     import torch
