@@ -15,6 +15,7 @@ Functions and their pins (tests/test_oracle_pins.py):
   kde            brute force (scipy pdist), closed form for coincident / two-point sets
   rdf            hand-computed shells, uniform-cube law (g -> 1 - O(r) boundary deficit)
   pairmatrix_hd  torch.cdist float64 on the decoded bf16 features, symmetry, diagonal
+  knn            lexsort brute force, lattice neighbour shells (6/12/8), index tie-break, k > n-1
 Parity status: no worked example in PAPER.md prints values, so every pin is a
 mathematical one; see DESIGN.md §Oracle.
 """
@@ -64,6 +65,8 @@ def _load():
         lib.oracle_rdf.argtypes = [_u64p, ctypes.c_int, ctypes.c_int, ctypes.c_double, _i64, ctypes.c_double, _f64p]
         lib.oracle_pairmatrix_hd.argtypes = [ctypes.POINTER(ctypes.c_uint16), _i64, ctypes.c_int, ctypes.c_int,
                                              ctypes.c_double, _i64, _i64, _f64p]
+        lib.oracle_knn.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_int, _i64, _i64,
+                                   ctypes.POINTER(ctypes.c_int64), _f64p]
         lib.oracle_num_threads.restype = ctypes.c_int
         _lib = lib
     return _lib
@@ -187,3 +190,16 @@ def pairmatrix_hd(features_bf16_bits, gamma, rows=None, ktype=0):
     if rc:
         raise ValueError(f"oracle_pairmatrix_hd: status {rc}")
     return out
+
+
+def knn(points, k, rows=None):
+    """All-point kNN: (idx int64 [rows, k], dist float64 [rows, k]) in (distance, index) order."""
+    p, n, dim = _pts(points)
+    rb, re = _rows(rows, n)
+    idx = np.zeros((re - rb, k), np.int64)
+    dist = np.zeros((re - rb, k), np.float64)
+    rc = _load().oracle_knn(_ptr(p, _f32p), n, dim, int(k), rb, re, idx.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                            _ptr(dist, _f64p))
+    if rc:
+        raise ValueError(f"oracle_knn: status {rc}")
+    return idx, dist

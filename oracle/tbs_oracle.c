@@ -303,3 +303,57 @@ int oracle_pairmatrix_hd(const uint16_t* X, int64_t n, int d, int ktype, double 
     }
   return ORACLE_OK;
 }
+
+/*
+ * All-point k-nearest neighbours (Type-I, NEXT-2 of SURVEY §8(f); PAPER.md L311-313:
+ * "all-point k-nearest neighbors (when k is small)", a Type-I output small enough for
+ * registers). For each anchor i in [row_begin, row_end): the k points j != i with the smallest
+ * Euclidean distance, in ascending (distance, j) order — equal distances go to the smaller
+ * index (reading R5). Written as the definition: scan j = 0 .. n-1, keep the k best so far
+ * sorted, and insert a candidate only if it is strictly better than the current k-th (an
+ * equal distance never displaces an earlier, smaller index). If n - 1 < k, the missing
+ * entries are idx -1, dist +inf. idx/dist are (row_end - row_begin) x k row-major.
+ */
+int oracle_knn(const float* P, int64_t n, int dim, int k, int64_t row_begin, int64_t row_end, int64_t* idx,
+               double* dist) {
+  if (check_common(P, n, dim, row_begin, row_end) || k < 1 || (row_end > row_begin && (!idx || !dist)))
+    return ORACLE_EINVAL;
+  int rc = ORACLE_OK;
+#pragma omp parallel
+  {
+    double* bs = (double*)malloc(sizeof(double) * (size_t)k);
+    int64_t* bj = (int64_t*)malloc(sizeof(int64_t) * (size_t)k);
+    if (!bs || !bj) {
+#pragma omp atomic write
+      rc = ORACLE_ENOMEM;
+    } else {
+#pragma omp for schedule(guided)
+      for (int64_t i = row_begin; i < row_end; ++i) {
+        for (int t = 0; t < k; ++t) {
+          bs[t] = INFINITY;
+          bj[t] = -1;
+        }
+        for (int64_t j = 0; j < n; ++j) {
+          if (j == i) continue;
+          const double s = dist2(P, dim, i, j);
+          if (!(s < bs[k - 1])) continue;
+          int t = k - 1;  /* shift worse entries down, insert after every entry <= s */
+          while (t > 0 && s < bs[t - 1]) {
+            bs[t] = bs[t - 1];
+            bj[t] = bj[t - 1];
+            --t;
+          }
+          bs[t] = s;
+          bj[t] = j;
+        }
+        for (int t = 0; t < k; ++t) {
+          idx[(i - row_begin) * k + t] = bj[t];
+          dist[(i - row_begin) * k + t] = sqrt(bs[t]);
+        }
+      }
+    }
+    free(bs);
+    free(bj);
+  }
+  return rc;
+}

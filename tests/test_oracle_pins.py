@@ -323,3 +323,71 @@ def test_pairmatrix_hd_vs_cdist():
     full = oracle.pairmatrix_hd(x, 0.3)
     assert np.array_equal(full, full.T) and np.all(np.diag(full) == 1.0)
     assert np.array_equal(oracle.pairmatrix_hd(x, 0.3, rows=(17, 90)), full[17:90])
+
+
+# ---- all-point kNN (NEXT-2; reading R5: ties -> smaller index) -----------
+def _knn_lexsort(p, k):
+    """Independent brute force: full distance matrix (scipy), then a lexicographic sort of
+    (distance, index) per row with the self pair removed."""
+    from scipy.spatial.distance import cdist
+    n = len(p)
+    D = cdist(p.astype(np.float64), p.astype(np.float64))
+    idx = np.full((n, k), -1, np.int64)
+    dist = np.full((n, k), np.inf)
+    for i in range(n):
+        j = np.array([x for x in range(n) if x != i], np.int64)
+        order = np.lexsort((j, D[i, j]))[:k]
+        idx[i, :len(order)] = j[order]
+        dist[i, :len(order)] = D[i, j[order]]
+    return idx, dist
+
+
+@pytest.mark.parametrize("dim,n,k,seed", [(1, 40, 3, 1), (2, 60, 5, 2), (3, 80, 8, 3), (4, 50, 16, 4), (3, 9, 12, 5)])
+def test_knn_vs_lexsort_bruteforce(dim, n, k, seed):
+    p = g.uniform(n, seed, dim)
+    i_o, d_o = oracle.knn(p, k)
+    i_b, d_b = _knn_lexsort(p, k)
+    assert np.array_equal(i_o, i_b)
+    np.testing.assert_allclose(d_o, d_b, rtol=1e-12, atol=0)
+
+
+def test_knn_lattice_neighbour_shells():
+    # unit cubic lattice: an interior point has 6 neighbours at 1, 12 at sqrt 2, 8 at sqrt 3;
+    # a corner has 3, 3, 1 (closed form)
+    L = 5
+    p = g.lattice(L, 11)
+    _, d = oracle.knn(p, 26)
+    key = [tuple(x) for x in p.astype(int)]
+    centre, corner = key.index((2, 2, 2)), key.index((0, 0, 0))
+    want = [1.0] * 6 + [math.sqrt(2)] * 12 + [math.sqrt(3)] * 8
+    np.testing.assert_allclose(d[centre], want, rtol=1e-15)
+    assert np.allclose(d[corner][:7], [1, 1, 1, math.sqrt(2), math.sqrt(2), math.sqrt(2), math.sqrt(3)])
+    assert d[corner][7] == 2.0
+    # every lattice point's nearest neighbour is at distance exactly 1
+    _, d1 = oracle.knn(p, 1)
+    assert np.all(d1[:, 0] == 1.0)
+
+
+def test_knn_ties_go_to_smaller_index():
+    p = np.zeros((7, 3), np.float32)               # all coincident: every distance is 0
+    idx, d = oracle.knn(p, 3)
+    for i in range(7):
+        assert list(idx[i]) == [j for j in range(7) if j != i][:3]
+    assert np.all(d == 0.0)
+    # two shells around point 0, inserted in scrambled index order
+    q = np.array([[0, 0, 0], [2, 0, 0], [1, 0, 0], [0, 2, 0], [0, 1, 0], [0, 0, 1]], np.float32)
+    idx, d = oracle.knn(q, 5)
+    assert list(idx[0]) == [2, 4, 5, 1, 3]
+    assert list(d[0]) == [1, 1, 1, 2, 2]
+
+
+def test_knn_k_exceeds_n_minus_1_and_rows():
+    p = g.uniform(4, 7, 3)
+    idx, d = oracle.knn(p, 6)
+    assert np.all(idx[:, 3:] == -1) and np.all(np.isinf(d[:, 3:]))
+    assert all(sorted(idx[i, :3]) == [j for j in range(4) if j != i] for i in range(4))
+    assert oracle.knn(np.zeros((1, 3), np.float32), 2)[0].tolist() == [[-1, -1]]
+    q = g.uniform(300, 8, 3)
+    full_i, full_d = oracle.knn(q, 4)
+    part_i, part_d = oracle.knn(q, 4, rows=(100, 170))
+    assert np.array_equal(part_i, full_i[100:170]) and np.array_equal(part_d, full_d[100:170])
