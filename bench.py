@@ -47,6 +47,7 @@ WORKLOADS = {
     "pairmatrix_64k": ("pairmatrix", "uniform", 1 << 16, 5, dict(gamma=1.0)),  # configs[4]
     "kde_uniform_1m": ("kde", "uniform", 1 << 20, 2, dict(gamma=1.0)),        # NEXT-2 (Type-I float sum)
     "pairmatrix_hd_64k_d64": ("pairmatrix_hd", "uniform", 1 << 16, 7, dict(d=64, gamma=1.0 / 64)),  # NEXT-3
+    "knn_uniform_1m_k8": ("knn", "uniform", 1 << 20, 2, dict(k=8)),  # NEXT-2 (all-point kNN)
     "pairmatrix_hd_64k_d512": ("pairmatrix_hd", "uniform", 1 << 16, 7, dict(d=512, gamma=1.0 / 512)),
 }
 METRIC = "SDH pair-distances/sec (G pairs/s) at N=1M–4M, 1/2/4/8 B200, % of roofline"
@@ -134,11 +135,14 @@ def oracle_rate(op, p, params, rows):
         oracle.kde(p, params["gamma"], rows=rows)
     elif op == "pairmatrix_hd":
         oracle.pairmatrix_hd(bf16_bits(p), params["gamma"], rows=rows)
+    elif op == "knn":
+        oracle.knn(p, params["k"], rows=rows)
     else:
         oracle.pairmatrix(p, params["gamma"], rows=rows)
     dt = time.perf_counter() - t0
     b, e = rows
-    units = (e - b) * n if op.startswith("pairmatrix") else (e - b) * (2 * n - b - e - 1) // 2
+    units = (e - b) * n if op.startswith("pairmatrix") else (e - b) * (n - 1) if op == "knn" else \
+        (e - b) * (2 * n - b - e - 1) // 2
     return units, dt
 
 
@@ -244,6 +248,10 @@ def main():
         out = torch.empty(1, dtype=torch.int64, device=dev)
     elif op == "kde":
         out = torch.empty(1, dtype=torch.float64, device=dev)
+    elif op == "knn":
+        rows_pm = (n * rank // world, n * (rank + 1) // world)
+        out = (torch.empty((rows_pm[1] - rows_pm[0], params["k"]), dtype=torch.int32, device=dev),
+               torch.empty((rows_pm[1] - rows_pm[0], params["k"]), dtype=torch.float32, device=dev))
     else:
         rows_pm = (n * rank // world, n * (rank + 1) // world)
         out = torch.empty((rows_pm[1] - rows_pm[0], n), dtype=torch.float32, device=dev)
@@ -259,6 +267,8 @@ def main():
             tbs.kde(pts, params["gamma"], out=out, events=events, group=pg)
         elif op == "pairmatrix_hd":
             tbs.pairmatrix_hd(pts, params["gamma"], out=out, events=events, group=pg)
+        elif op == "knn":
+            tbs.knn(pts, params["k"], out=out, events=events, group=pg)
         else:
             tbs.pairmatrix(pts, params["gamma"], out=out, events=events, group=pg)
 
@@ -300,7 +310,7 @@ def main():
         kavg = sum(kms) / len(kms)
 
     is_matrix = op in ("pairmatrix", "pairmatrix_hd")
-    units = units_of("pairmatrix" if is_matrix else "sdh", n)
+    units = units_of("pairmatrix" if is_matrix else "sdh", n) * (2 if op == "knn" else 1)  # kNN: ordered pairs
     value = units * args.steps / (ms * 1e-3) / 1e9
     unit = "G pairs/s" if not is_matrix else "G entries/s"
     pk = peaks()
@@ -330,8 +340,14 @@ def main():
     else:
         rb, re = tbs.rank_rows(n, world, rank)
         rank_units = (re - rb) * (2 * n - rb - re - 1) // 2
+        if op == "knn":
+            rb, re = n * rank // world, n * (rank + 1) // world
+            rank_units = (re - rb) * (n - 1)
         pairs_s = rank_units / (kavg * 1e-3)
-        if op == "pcf":
+        if op == "knn":
+            peak = pk["fp32"] / 6
+            bound_note = "FP32 pipe: 6 lane-ops per ordered pair (3 sub + 3 mul/fma); compare + rare insert on ALU"
+        elif op == "pcf":
             peak = pk["fp32"] / 6
             bound_note = "FP32 pipe: 6 lane-ops/pair (3 sub + 3 mul/fma)"
         elif op == "kde":
@@ -358,7 +374,7 @@ def main():
 
     # e2e: host buffers through the public API, H2D of the points and D2H of the result each step
     e2e = None
-    if op in ("sdh", "pcf", "kde"):
+    if op in ("sdh", "pcf", "kde", "knn"):
         ph = torch.from_numpy(p_host).pin_memory()
         if world == 1:
             hh = np.zeros(nb if op == "sdh" else 1, np.uint64)
@@ -369,10 +385,12 @@ def main():
                     tbs.sdh_host(ph.numpy(), w, nb, out=hh)
                 elif op == "kde":
                     tbs.lib().tbs_kde(ph.numpy().ctypes.data, n, ctypes.c_float(params["gamma"]), kh.ctypes.data)
+                elif op == "knn":
+                    tbs.knn_host(ph.numpy(), params["k"])
                 else:
                     tbs.pcf_host(ph.numpy(), params["r"])
         else:
-            res_h = torch.empty(out.shape, dtype=out.dtype).pin_memory()
+            res_h = torch.empty((out[1] if op == "knn" else out).shape, dtype=(out[1] if op == "knn" else out).dtype).pin_memory()
 
             def e2e_step():
                 d = ph.to(dev, non_blocking=True)
@@ -380,6 +398,8 @@ def main():
                     r = tbs.sdh(d, w, nb, group=pg)
                 elif op == "kde":
                     r = tbs.kde(d, params["gamma"], group=pg)
+                elif op == "knn":
+                    r = tbs.knn(d, params["k"], group=pg)[1]
                 else:
                     r = tbs.pcf(d, params["r"], group=pg)
                 res_h.copy_(r)
@@ -398,8 +418,9 @@ def main():
             tt = torch.tensor([te], dtype=torch.float64, device=dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             te = tt.item()
+        d2h = int(out[0].numel() * 8) if op == "knn" else int(out.numel() * 8)
         e2e = {"value": units * ke / te / 1e9, "unit": unit, "h2d_bytes_per_step": int(p_host.nbytes),
-               "d2h_bytes_per_step": int(out.numel() * 8)}
+               "d2h_bytes_per_step": d2h}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

@@ -120,6 +120,20 @@ int tbs_pairmatrix_ex(const tbs_args* args, tbs_kernel kernel, float* out);
 int tbs_kde(const float* points, int64_t n, float gamma, double* sum);
 int tbs_kde_ex(const tbs_args* args, float gamma, double* sum);   /* sum: device, overwritten */
 
+/* All-point k-nearest neighbours, a Type-I 2-BS ("all-point k-nearest
+ * neighbors (when k is small)"; reading R5). For every anchor i (all i in [0, n) for
+ * tbs_knn; i in [row_begin, row_end) for tbs_knn_ex), the k points j != i of smallest Euclidean
+ * distance, ascending by (fp32 squared distance, j): equal distances list the smaller index
+ * first. Row r = i - row_begin: idx[r*k + t] (int32, j) and dist[r*k + t] (fp32, the correctly
+ * rounded sqrt of the fp32 squared distance), t = 0..k-1; if n - 1 < k the missing entries are
+ * idx -1, dist +inf. 1 <= k <= TBS_KNN_MAX_K; coordinates must be finite.
+ * tbs_knn: points[n][dim] and idx/dist host or device (all alike), synchronous.
+ * tbs_knn_ex: device pointers, enqueued on args->stream; ev_begin/ev_end bracket the kNN
+ * kernel and its segment merge. Scratch is stream-ordered and freed on return. */
+#define TBS_KNN_MAX_K 32
+int tbs_knn(const float* points, int64_t n, int dim, int k, int32_t* idx, float* dist);
+int tbs_knn_ex(const tbs_args* args, int k, int32_t* idx, float* dist);
+
 /* Radial distribution function, "a normalized form of SDH": host arrays,
  * g[k] = hist[k] / (C(n,2) * shell_k / volume), shell_k the dim-ball shell volume between
  * k w and (k+1) w (no periodic boundary). Host-only arithmetic on an SDH result. */

@@ -12,6 +12,7 @@ library or a CUDA device is missing, calls raise.
     pairmatrix(points, gamma=1.0)         Type-III Gaussian pair matrix      (float32[rows, n])
     rank_rows(n, world, rank)             pair-balanced anchor-row partition
     kde(points, gamma)                    Type-I kernel-density pair sum      (float64[1])   (NEXT-2)
+    knn(points, k)                        Type-I all-point k nearest neighbours (int32, float32 [n, k]) (NEXT-2)
     rdf(points, bucket_width, nb, volume) radial distribution function       (float64[nb])  (NEXT-1)
     sdh_host / pcf_host / pairmatrix_host the same through host (numpy) buffers
 """
@@ -38,7 +39,7 @@ HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "
 
 # Symbols declared in include/tbs.h (checked by tests/test_abi.py).
 EXPORTS = ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
-           "tbs_kde", "tbs_kde_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex",
+           "tbs_kde", "tbs_kde_ex", "tbs_knn", "tbs_knn_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex",
            "tbs_rank_rows", "tbs_last_error", "tbs_release", "tbs_launch_count", "tbs_version")
 
 
@@ -75,6 +76,8 @@ def lib() -> ctypes.CDLL:
         L.tbs_pairmatrix_ex.argtypes = [ctypes.POINTER(_Args), _Kernel, vp]
         L.tbs_kde.argtypes = [vp, i64, ctypes.c_float, vp]
         L.tbs_kde_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_float, vp]
+        L.tbs_knn.argtypes = [vp, i64, ctypes.c_int, ctypes.c_int, vp, vp]
+        L.tbs_knn_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_int, vp, vp]
         L.tbs_rdf.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_float, i64, ctypes.c_double, vp]
         L.tbs_pairmatrix_hd.argtypes = [vp, i64, ctypes.c_int, _Kernel, vp]
         L.tbs_pairmatrix_hd_ex.argtypes = [vp, i64, ctypes.c_int, i64, i64, _Kernel, vp, vp, vp, vp]
@@ -84,7 +87,7 @@ def lib() -> ctypes.CDLL:
         L.tbs_launch_count.restype = ctypes.c_uint64
         L.tbs_release.restype = None
         for f in ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
-                  "tbs_kde", "tbs_kde_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex", "tbs_rank_rows", "tbs_version"):
+                  "tbs_kde", "tbs_kde_ex", "tbs_knn", "tbs_knn_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex", "tbs_rank_rows", "tbs_version"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -197,6 +200,28 @@ def kde(points, gamma: float, *, rows=None, out=None, stream=None, events=None, 
     return combine(s, group)
 
 
+def knn(points, k: int, *, rows=None, out=None, stream=None, events=None, group=None):
+    """All-point k nearest neighbours (Type-I, NEXT-2): for each anchor row, the k nearest other
+    points in ascending (distance, index) order. Returns (idx int32 [rows, k], dist float32
+    [rows, k]); missing entries (n - 1 < k) are (-1, inf). With a group each rank computes an
+    equal block of anchor rows (every row costs n - 1 distances); no collective is needed."""
+    torch = _torch()
+    n = points.shape[0]
+    if group is not None:
+        import torch.distributed as dist
+        W, r = dist.get_world_size(group), dist.get_rank(group)
+        rows = (n * r // W, n * (r + 1) // W)
+    a, _ = _args(points, rows, 0, stream, events)
+    nr = a.row_end - a.row_begin
+    if out is not None:
+        idx, dist_ = out
+    else:
+        idx = torch.empty((nr, k), dtype=torch.int32, device=points.device)
+        dist_ = torch.empty((nr, k), dtype=torch.float32, device=points.device)
+    _check(lib().tbs_knn_ex(ctypes.byref(a), int(k), idx.data_ptr(), dist_.data_ptr()), "tbs_knn_ex")
+    return idx, dist_
+
+
 def rdf_from_hist(hist, bucket_width: float, n: int, volume: float, dim: int = 3):
     """RDF g[k] (NEXT-1) from an SDH histogram (host arithmetic in libtbs: tbs_rdf)."""
     h = np.ascontiguousarray(hist.cpu().numpy() if hasattr(hist, "cpu") else hist).astype(np.uint64)
@@ -285,3 +310,13 @@ def pairmatrix_host(points, gamma: float = 1.0, kernel: str = "gaussian"):
     _check(lib().tbs_pairmatrix(p.ctypes.data, n, _Kernel(KERNELS[kernel], float(gamma)), o.ctypes.data),
            "tbs_pairmatrix")
     return o
+
+
+def knn_host(points, k: int):
+    """tbs_knn with host buffers: (idx int32 [n, k], dist float32 [n, k])."""
+    p = _host_points(points)
+    n = p.shape[0]
+    idx = np.empty((n, k), np.int32)
+    d = np.empty((n, k), np.float32)
+    _check(lib().tbs_knn(p.ctypes.data, n, p.shape[1], int(k), idx.ctypes.data, d.ctypes.data), "tbs_knn")
+    return idx, d

@@ -18,6 +18,7 @@
 #include "tbs.h"
 #include "tbs_kernels.cuh"
 #include "tbs_hd.cuh"
+#include "tbs_knn.cuh"
 
 using namespace tbs;
 
@@ -218,7 +219,7 @@ int validate_common(const tbs_args* a) {
 // SoA copy of the points in stream-ordered scratch; the loader also zeroes `zero` words.
 // The allocation holds SoA [D][n_pad] followed by the 2D+1 bounding-box words.
 int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long long* zero, long long zero_words,
-                cudaStream_t st, uint32_t** bbox) {
+                cudaStream_t st, uint32_t** bbox, float pad = 0.0f) {
   const size_t soa_bytes = (size_t)D * n_pad * sizeof(float);
   TBS_CUDA(cudaMallocAsync((void**)soa, soa_bytes + 64, st));
   *bbox = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(*soa) + soa_bytes);
@@ -226,8 +227,8 @@ int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long 
   const int threads = 256;
   long long blocks = std::min<long long>((n_pad + threads - 1) / threads, 148ll * 16);
   blocks = std::max<long long>(blocks, 1);
-  soa_loader<<<(unsigned)blocks, threads, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, D, *soa, zero, zero_words,
-                                                   *bbox);
+  soa_loader<<<(unsigned)blocks, threads, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, D, pad, *soa, zero,
+                                                   zero_words, *bbox);
   TBS_CUDA(cudaGetLastError());
   g_launches.fetch_add(1);
   return TBS_OK;
@@ -646,6 +647,78 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
   return rc;
 }
 
+// ---- NEXT-2: all-point kNN ---------------------------------------------------------------
+template <int K, int KA, int D>
+int knn_launch(const Device& dev, const tbs_args* a, const float* soa, int n_pad, int k, int32_t* idx, float* dist,
+               cudaStream_t st) {
+  constexpr int TA = knn::kThreads * KA;
+  auto kern = knn::knn_kernel<K, KA, D>;
+  static thread_local int occ_dev = -1, occ = 0;
+  if (occ_dev != dev.id) {
+    TBS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, knn::kThreads, 0));
+    occ_dev = dev.id;
+  }
+  const int n = (int)a->n, rb = (int)a->row_begin, re = (int)a->row_end, rows = re - rb;
+  const int I0 = rb / TA, tiles = (re + TA - 1) / TA - I0;
+  const int n_chunks = (n + knn::kTP - 1) / knn::kTP;
+  // partner segments so the grid is >= ~8 waves (wave-quantisation loss <= 1/8)
+  const long long slots = (long long)dev.sms * std::max(occ, 1);
+  int S = (int)std::min<long long>(std::max<long long>(1, (8 * slots + tiles - 1) / tiles), n_chunks);
+  const int seg = (n_chunks + S - 1) / S;
+  S = (n_chunks + seg - 1) / seg;
+  float* ps = nullptr;
+  int* pj = nullptr;
+  if (S > 1) {
+    TBS_CUDA(cudaMallocAsync((void**)&ps, (size_t)S * rows * K * 8, st));
+    pj = reinterpret_cast<int*>(ps + (size_t)S * rows * K);
+  }
+  cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
+  int rc = TBS_OK;
+  if (eb) TBS_CUDA(cudaEventRecord(eb, st));
+  kern<<<dim3((unsigned)tiles, (unsigned)S), knn::kThreads, 0, st>>>(soa, n, n_pad, rb, re, I0, seg, n_chunks, k, ps, pj,
+                                                                     idx, dist);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) rc = fail(TBS_ECUDA, "knn_kernel: %s", cudaGetErrorString(e));
+  g_launches.fetch_add(1);
+  if (!rc && S > 1) {
+    knn::knn_merge<K><<<(unsigned)((rows + 127) / 128), 128, 0, st>>>(ps, pj, rows, S, k, idx, dist);
+    e = cudaGetLastError();
+    if (e != cudaSuccess) rc = fail(TBS_ECUDA, "knn_merge: %s", cudaGetErrorString(e));
+    g_launches.fetch_add(1);
+  }
+  if (!rc && ee) TBS_CUDA(cudaEventRecord(ee, st));
+  if (ps) cudaFreeAsync(ps, st);
+  return rc;
+}
+
+int knn_impl(const tbs_args* a, int k, int32_t* idx, float* dist) {
+  int rc = validate_common(a);
+  if (rc) return rc;
+  if (k < 1 || k > TBS_KNN_MAX_K) return fail(TBS_EINVAL, "k = %d outside [1, %d]", k, TBS_KNN_MAX_K);
+  if (a->row_end > a->row_begin && (!idx || !dist)) return fail(TBS_EINVAL, "idx or dist is NULL");
+  if (a->row_end == a->row_begin) return TBS_OK;
+  Device dev;
+  if ((rc = current_device(dev))) return rc;
+  cudaStream_t st = (cudaStream_t)a->stream;
+  const int D = a->dim <= 3 ? 3 : 4;
+  const int n_pad = pad_rows(a->n);
+  float* soa = nullptr;
+  uint32_t* bbox = nullptr;
+  rc = load_points(a, D, n_pad, &soa, nullptr, 0, st, &bbox, INFINITY);
+  if (!rc) {
+    if (D == 3) rc = k <= 4 ? knn_launch<4, 4, 3>(dev, a, soa, n_pad, k, idx, dist, st)
+                     : k <= 8 ? knn_launch<8, 4, 3>(dev, a, soa, n_pad, k, idx, dist, st)
+                     : k <= 16 ? knn_launch<16, 2, 3>(dev, a, soa, n_pad, k, idx, dist, st)
+                               : knn_launch<32, 2, 3>(dev, a, soa, n_pad, k, idx, dist, st);
+    else rc = k <= 4 ? knn_launch<4, 4, 4>(dev, a, soa, n_pad, k, idx, dist, st)
+              : k <= 8 ? knn_launch<8, 4, 4>(dev, a, soa, n_pad, k, idx, dist, st)
+              : k <= 16 ? knn_launch<16, 2, 4>(dev, a, soa, n_pad, k, idx, dist, st)
+                        : knn_launch<32, 2, 4>(dev, a, soa, n_pad, k, idx, dist, st);
+  }
+  if (soa) cudaFreeAsync(soa, st);
+  return rc;
+}
+
 // ---- host-or-device simple entry points ------------------------------------------
 int is_device_ptr(const void* p, bool& dev) {
   dev = false;
@@ -813,6 +886,37 @@ int tbs_pairmatrix_hd(const uint16_t* features, int64_t n, int d, tbs_kernel ker
   cudaFreeAsync(dout, st);
   e = cudaStreamSynchronize(st);
   if (!rc && e != cudaSuccess) rc = fail(TBS_ECUDA, "sync: %s", cudaGetErrorString(e));
+  return rc;
+}
+
+int tbs_knn_ex(const tbs_args* args, int k, int32_t* idx, float* dist) {
+  g_err.clear();
+  return knn_impl(args, k, idx, dist);
+}
+
+int tbs_knn(const float* points, int64_t n, int dim, int k, int32_t* idx, float* dist) {
+  g_err.clear();
+  if (n < 0 || n > TBS_MAX_N || k < 1 || k > TBS_KNN_MAX_K || !idx || !dist)
+    return fail(TBS_EINVAL, "tbs_knn: bad arguments");
+  const size_t half = (size_t)n * (size_t)k * 4;
+  bool ddev = false;
+  is_device_ptr(dist, ddev);
+  if (ddev) {
+    bool idev = false;
+    is_device_ptr(idx, idev);
+    if (!idev) return fail(TBS_EINVAL, "idx and dist must both be host or both device pointers");
+    return run_simple(points, n, dim, dist, half, [&](tbs_args* a, void*) { return knn_impl(a, k, idx, dist); });
+  }
+  // host buffers: one device allocation holds [idx | dist]; copy both halves back
+  std::vector<unsigned char> both(2 * half + 4);
+  int rc = run_simple(points, n, dim, both.data(), 2 * half + 4, [&](tbs_args* a, void* o) {
+    return knn_impl(a, k, reinterpret_cast<int32_t*>(o),
+                    reinterpret_cast<float*>(reinterpret_cast<unsigned char*>(o) + half));
+  });
+  if (!rc && half) {
+    std::memcpy(idx, both.data(), half);
+    std::memcpy(dist, both.data() + half, half);
+  }
   return rc;
 }
 

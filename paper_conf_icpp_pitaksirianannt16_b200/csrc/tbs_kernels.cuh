@@ -87,14 +87,16 @@ __device__ __forceinline__ float ord2f(uint32_t o) {
   return __uint_as_float((o & 0x80000000u) ? (o & 0x7fffffffu) : ~o);
 }
 
-__global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_pad, int D,
+// `pad` is the coordinate value of pad points i >= n (0; +inf for kNN, so pad partners never
+// enter a neighbour list).
+__global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_pad, int D, float pad,
                            float* __restrict__ soa, unsigned long long* __restrict__ zero, long long zero_words,
                            uint32_t* __restrict__ bbox) {
   const long long stride = (long long)gridDim.x * blockDim.x;
   uint32_t lo[4] = {0u, 0u, 0u, 0u}, hi[4] = {0u, 0u, 0u, 0u}, bad = 0u;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n_pad; i += stride) {
     for (int c = 0; c < D; ++c) {
-      float v = 0.0f;
+      float v = i < n ? 0.0f : pad;
       if (i < n && c < dim) {
         v = __ldg(pts + i * dim + c);
         const uint32_t o = f2ord(v);

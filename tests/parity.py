@@ -1,5 +1,6 @@
 """Acceptance rules for GPU-vs-oracle parity (BASELINE.json north star)."""
 import numpy as np
+import oracle
 
 
 def check_sdh_float(h_gpu, h_or, amb):
@@ -36,3 +37,28 @@ def check_matrix(out_gpu, out_or, rtol=1e-5):
     m = float(rel.max()) if rel.size else 0.0
     assert m <= rtol, f"max rel err {m}"
     return m
+
+
+def check_knn_float(p, k, gi, gd, rows=None, rtol=4e-6):
+    """Float inputs: the GPU orders by the fp32 squared distance, so near-ties may swap.
+    Checks: distances agree with the oracle's position by position (rtol); every returned
+    index is valid, distinct, not the anchor, and its true distance equals the reported one;
+    where the oracle's distance at a position is separated from its neighbours by more than
+    the tolerance, the index is the oracle's."""
+    oi, od = oracle.knn(p, k, rows=rows)
+    rb = 0 if rows is None else rows[0]
+    fin = np.isfinite(od)
+    assert np.array_equal(np.isfinite(gd), fin) and np.all(gi[~fin] == -1)
+    np.testing.assert_allclose(gd[fin], od[fin], rtol=rtol, atol=1e-30)
+    P = p.astype(np.float64)
+    for r in range(len(gi)):
+        row = gi[r][gi[r] >= 0]
+        assert len(set(row.tolist())) == len(row) and (rb + r) not in row
+        true = np.sqrt(((P[row] - P[rb + r]) ** 2).sum(1))
+        np.testing.assert_allclose(gd[r][:len(row)], true, rtol=rtol, atol=1e-30)
+        sep = np.ones(k, bool)
+        dd = od[r]
+        gap = rtol * 4 * np.maximum(dd, 1e-30)
+        sep[1:] &= (dd[1:] - dd[:-1]) > gap[1:]
+        sep[:-1] &= (dd[1:] - dd[:-1]) > gap[:-1]
+        assert np.array_equal(gi[r][sep & fin[r]], oi[r][sep & fin[r]]), r

@@ -16,7 +16,7 @@ import pytest
 
 import oracle
 import tbs_inputs as g
-from parity import check_matrix, check_pcf_float, check_sdh_float
+from parity import check_knn_float, check_matrix, check_pcf_float, check_sdh_float
 
 pytestmark = pytest.mark.gpu
 GOLD = os.path.join(os.path.dirname(__file__), "golden")
@@ -187,3 +187,27 @@ def test_pairmatrix_hd_64k_sampled_rows(tbs):
         ref = oracle.pairmatrix_hd(xb, 1.0 / d, rows=(r, r + 1))[0]
         B = 2.0 ** -23 * (d / 16 + 8) * (nrm[r] + nrm + 2 * np.abs(xf) @ np.abs(xf[r]))
         assert np.all(np.abs(got[k] - ref) <= ref * (g32 * B + 2e-6)), r
+
+
+# ---------------------------------------------------------------- NEXT-2: kNN at the bench size
+def test_knn_1m_sampled_strips(tbs):
+    """bench.py knn_uniform_1m_k8: 1M uniform points, k = 8 (3 partner segments + merge)."""
+    n, k = 1 << 20, 8
+    p = g.uniform(n, 2)
+    i, d = tbs.knn(dev(p), k)
+    gi, gd = host(i).astype(np.int64), host(d)
+    for rb, re in strips(n, 16):
+        check_knn_float(p, k, gi[rb:re], gd[rb:re], rows=(rb, re))
+
+
+def test_knn_lattice_2_5m_exact_strips(tbs):
+    """137^3 = 2.57M lattice points: enough anchor tiles for the single-segment path
+    (direct output, no merge); bit-exact against the oracle on strips."""
+    L, k = 137, 16
+    p = g.lattice(L, 5)
+    n = len(p)
+    i, d = tbs.knn(dev(p), k)
+    gi, gd = host(i).astype(np.int64), host(d)
+    for rb, re in strips(n, 8):
+        oi, od = oracle.knn(p, k, rows=(rb, re))
+        assert np.array_equal(gi[rb:re], oi) and np.array_equal(gd[rb:re], od.astype(np.float32))

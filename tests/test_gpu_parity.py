@@ -17,7 +17,7 @@ import pytest
 
 import oracle
 import tbs_inputs as g
-from parity import check_matrix, check_pcf_float, check_sdh_float
+from parity import check_knn_float, check_matrix, check_pcf_float, check_sdh_float
 
 pytestmark = pytest.mark.gpu
 
@@ -387,3 +387,68 @@ def test_pairmatrix_hd_rows_and_host(tbs):
     assert np.array_equal(host, full)
     ref = oracle.pairmatrix_hd(xb, 0.01)
     assert np.all(np.abs(full - ref) <= ref * (0.01 * _hd_bound(xb) + 2e-6))
+
+
+# ------------------------------------------------------------------ NEXT-2: all-point kNN (reading R5)
+def knn_gpu(tbs, p, k, rows=None):
+    import torch
+    i, d = tbs.knn(dev(p), k, rows=rows)
+    torch.cuda.synchronize()
+    return i.cpu().numpy().astype(np.int64), d.cpu().numpy()
+
+
+@pytest.mark.parametrize("L,cut,k", [(12, None, 1), (12, None, 6), (12, None, 8), (12, None, 13), (12, None, 26),
+                                     (16, 3001, 4), (16, 4095, 16), (20, 7777, 32), (10, 1000, 18)])
+def test_knn_lattice_exact(tbs, L, cut, k):
+    """Integer lattice: squared distances exact in fp32, so idx and dist are bit-exact,
+    including the smaller-index-first rule on the many lattice ties."""
+    p = g.lattice(L, 30 + L)[:cut]
+    oi, od = oracle.knn(p, k)
+    gi, gd = knn_gpu(tbs, p, k)
+    assert np.array_equal(gi, oi)
+    assert np.array_equal(gd, od.astype(np.float32))
+
+
+@pytest.mark.parametrize("kind,n,k", [("uniform", 3000, 1), ("uniform", 5000, 5), ("clustered", 9000, 8),
+                                      ("clustered", 4097, 16), ("uniform", 12345, 32), ("uniform", 20000, 3)])
+def test_knn_float(tbs, kind, n, k):
+    p = g.make(kind, n, 50 + n)
+    gi, gd = knn_gpu(tbs, p, k)
+    check_knn_float(p, k, gi, gd)
+
+
+def test_knn_rows_dims_and_edges(tbs):
+    p = g.lattice(14, 3)[:2700]
+    oi, od = oracle.knn(p, 7)
+    parts = [knn_gpu(tbs, p, 7, rows=(2700 * r // 4, 2700 * (r + 1) // 4)) for r in range(4)]
+    assert np.array_equal(np.concatenate([x[0] for x in parts]), oi)
+    assert np.array_equal(np.concatenate([x[1] for x in parts]), od.astype(np.float32))
+    gi, gd = knn_gpu(tbs, p, 7, rows=(1000, 1013))
+    assert np.array_equal(gi, oi[1000:1013])
+    for dim in (1, 2, 4):
+        q = g.uniform(3000, 90 + dim, dim)
+        gi, gd = knn_gpu(tbs, q, 6)
+        check_knn_float(q, 6, gi, gd)
+    # coincident points: every distance 0, ties by index
+    z = np.zeros((300, 3), np.float32)
+    gi, gd = knn_gpu(tbs, z, 5)
+    assert np.array_equal(gi, oracle.knn(z, 5)[0]) and np.all(gd == 0)
+    # k > n - 1, n = 1, n = 0
+    q = g.uniform(5, 4)
+    gi, gd = knn_gpu(tbs, q, 9)
+    oi, od = oracle.knn(q, 9)
+    assert np.array_equal(gi, oi) and np.all(np.isinf(gd[:, 4:]))
+    gi, gd = knn_gpu(tbs, q[:1], 3)
+    assert gi.tolist() == [[-1, -1, -1]] and np.all(np.isinf(gd))
+    assert knn_gpu(tbs, q[:0], 3)[0].shape == (0, 3)
+
+
+def test_knn_host_entry_point_and_einval(tbs):
+    p = g.lattice(9, 5)
+    gi, gd = tbs.knn_host(p, 10)
+    oi, od = oracle.knn(p, 10)
+    assert np.array_equal(gi.astype(np.int64), oi) and np.array_equal(gd, od.astype(np.float32))
+    with pytest.raises(tbs.TbsError):
+        tbs.knn(dev(p), 33)
+    with pytest.raises(tbs.TbsError):
+        tbs.knn(dev(p), 0)
