@@ -16,7 +16,7 @@
 //     into shared memory by the producer beside the operands), apply the kernel (ex2 for the
 //     Gaussian), stage the tile in shared memory, and write it with coalesced streaming
 //     16-byte stores (each warp row = 512 contiguous bytes).
-// A dedicated producer warp overlaps the next tile's loads + MMAs with the epilogue.
+// A TMA producer warp and an MMA-issuer warp overlap the next tile's loads + MMAs with the epilogue.
 #pragma once
 #include <cstdint>
 #include "tbs_ptx.cuh"
@@ -29,10 +29,11 @@ constexpr int kKBlock = 64;         // bf16 per 128-byte swizzle row (one TMA bo
 constexpr int kRing = 4;            // operand ring: 4 stages of (A, B) k-blocks = 128 KB
 constexpr int kMaxD = 1024;         // feature dimension limit (k-blocks stream through the ring)
 constexpr int kEpiWarps = 16;                    // 4 TMEM lane quarters x 4 column chunks of 32
-constexpr int kThreads = (kEpiWarps + 1) * 32;   // + one producer / MMA warp
+constexpr int kThreads = (kEpiWarps + 2) * 32;   // + a TMA producer warp and an MMA warp
 constexpr int kStageBytes = kTile * kKBlock * 2; // 16 KB
 constexpr int kBoxCols = 32;                     // output TMA box: 128 rows x 32 fp32 (128 B, SWIZZLE_128B)
 constexpr int kTmemCols = 256;                   // two 128-column fp32 accumulators
+constexpr int kBand = 16;                        // tile rows per raster band
 
 struct Smem {
   // offsets from the 1024-aligned dynamic smem base
@@ -71,6 +72,30 @@ __device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t a_desc, uint64_
       "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
       "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)
       : "memory");
+}
+// One k-block of 64 = four K=16 MMAs (descriptors advance 32 B = 2 units per K step) and the
+// commit of the operand stage, in ONE asm block issued by one elected lane of a warp-uniform
+// loop: per-instruction elect/uniform-register overhead would otherwise make the issuing
+// thread slower than the tensor pipe (measured: ~115 SASS instructions per k-block).
+__device__ __forceinline__ void tc_mma_kblock(uint32_t d_tmem, uint64_t a_desc, uint64_t b_desc, uint32_t idesc,
+                                              uint32_t accumulate, uint32_t bar) {
+  asm volatile(
+      "{\n.reg .pred p;\n.reg .b64 a1, a2, a3, b1, b2, b3;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "add.s64 a1, %1, 2;\nadd.s64 a2, %1, 4;\nadd.s64 a3, %1, 6;\n"
+      "add.s64 b1, %2, 2;\nadd.s64 b2, %2, 4;\nadd.s64 b3, %2, 6;\n"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], a1, b1, %3, 1;\n"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], a2, b2, %3, 1;\n"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], a3, b3, %3, 1;\n"
+      "tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%5];\n}\n" ::"r"(d_tmem),
+      "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate), "r"(bar)
+      : "memory");
+}
+__device__ __forceinline__ bool elect_one() {
+  uint32_t e;
+  asm volatile("{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\nselp.u32 %0, 1, 0, p;\n}\n" : "=r"(e));
+  return e != 0u;
 }
 // TMA 1-D bulk store shared -> global (bulk async-group completion), used to drain the
 // staged output tile without occupying the warps (SASS: UBLKCP).
@@ -188,8 +213,30 @@ __global__ void __launch_bounds__(kThreads, 1)
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(sm + Smem::TMEM);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const long long ntiles = (long long)tiles_i * tiles_j;
-  // contiguous tile range per CTA (row-major: consecutive tiles share the row block I)
-  const long long t_beg = ntiles * blockIdx.x / gridDim.x, t_end = ntiles * (blockIdx.x + 1) / gridDim.x;
+  // Operand-heavy shapes (kblocks > 2): tiles are dealt round-robin (CTA b takes tiles b,
+  // b + grid, ...), so the grid works on ~grid consecutive tiles at a time, and consecutive
+  // tiles follow a grouped raster: bands of kBand tile rows walked column by column. The tiles
+  // in flight then share a few B column blocks and one A band (L2 hits; DRAM operand reads
+  // 7.2 GB -> 2.1 GB at 64K x 512). Output-bound shapes (small d) keep a contiguous row-major
+  // range per CTA (each CTA streams whole output rows: measured faster at d = 64).
+  const bool banded = kblocks > 2;
+  const long long c_beg = ntiles * blockIdx.x / gridDim.x;
+  const long long my_tiles = banded ? (ntiles > blockIdx.x ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0)
+                                    : ntiles * (blockIdx.x + 1) / gridDim.x - c_beg;
+  auto tile_ij = [&](long long k, int& I, int& J) {
+    if (!banded) {
+      const long long t = c_beg + k;
+      I = I0 + (int)(t / tiles_j);
+      J = (int)(t % tiles_j);
+      return;
+    }
+    const long long t = (long long)blockIdx.x + k * gridDim.x;
+    const long long band = t / ((long long)kBand * tiles_j);
+    const long long w = t - band * kBand * tiles_j;
+    const int rows = min(kBand, tiles_i - (int)band * kBand);
+    I = I0 + (int)band * kBand + (int)(w % rows);
+    J = (int)(w / rows);
+  };
 
   if (warp == kEpiWarps) {
     if (lane == 0) {
@@ -221,57 +268,61 @@ __global__ void __launch_bounds__(kThreads, 1)
   const uint32_t tmem = *tmem_holder;
 
   if (warp == kEpiWarps) {
-    if (lane == 0) {
-      // Producer / MMA issuer. Every wait below is on the completion right after the last
-      // one this thread consumed for that barrier, so no barrier can run two phases ahead.
-      const uint64_t keep = policy_evict_last();
-      // Operand k-blocks of consecutive tiles stream through a kRing-deep ring; loads run up
-      // to kRing k-blocks ahead of the MMAs. A tile's norms go into a 4-slot ring with its
-      // first k-block.
-      const long long total = (t_end - t_beg) * (long long)kblocks;
-      long long gl = 0;                                   // next k-block to load
-      auto load_next = [&]() {
-        const int st = (int)(gl % kRing);
-        if (gl >= kRing) mbar_wait(bar_free(st), (uint32_t)(((gl / kRing) - 1) & 1));   // MMAs of gl-kRing done
-        const long long ti = gl / kblocks;
-        const int kb = (int)(gl % kblocks);
-        const long long t = t_beg + ti;
-        const int I = I0 + (int)(t / tiles_j), J = (int)(t % tiles_j);
-        if (kb == 0) {
-          const int ns = (int)(ti & 3);
-          if (ti >= 4) mbar_wait(bar_nempty(ns), (uint32_t)(((ti - 4) >> 2) & 1));      // epilogue of ti-4 read slot
-          mbar_arrive_expect_tx(bar_nfull(ns), 2 * kTile * 4);
-          const uint32_t nd = sbase + Smem::NORMS + ns * 2 * kTile * 4;
-          bulk_g2s(nd, norms + I * kTile, kTile * 4, bar_nfull(ns));
-          bulk_g2s(nd + kTile * 4, norms + J * kTile, kTile * 4, bar_nfull(ns));
-        }
-        mbar_arrive_expect_tx(bar_full(st), (uint32_t)(2 * kStageBytes));
-        const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
-        // features stay L2-resident (evict_last) under the output stream
-        tma_load_2d_hint(ops, &tmap, kb * kKBlock, I * kTile, bar_full(st), keep);
-        tma_load_2d_hint(ops + kStageBytes, &tmap, kb * kKBlock, J * kTile, bar_full(st), keep);
-        ++gl;
-      };
-      int it = 0;
-      for (long long t = t_beg; t < t_end; ++t, ++it) {
-        const int acc = it & 1;
-        const uint32_t d_tmem = tmem + (uint32_t)(acc * kTile);
-        for (int kb = 0; kb < kblocks; ++kb) {
-          const long long gm = (long long)it * kblocks + kb;   // k-block consumed now
-          while (gl < total && gl < gm + kRing) load_next();
-          const int st = (int)(gm % kRing);
-          mbar_wait(bar_full(st), (uint32_t)((gm / kRing) & 1));
-          if (kb == 0 && it >= 2) mbar_wait(bar_acc_empty(acc), (uint32_t)(((it - 2) >> 1) & 1));  // acc drained
-          tc_fence_after();
-          const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
-#pragma unroll
-          for (int ks = 0; ks < kKBlock / 16; ++ks)
-            tc_mma(d_tmem, sw128_desc(ops + ks * 32), sw128_desc(ops + kStageBytes + ks * 32), kIdesc,
-                   (kb | ks) != 0 ? 1u : 0u);
-          tc_commit(bar_free(st));
-        }
-        tc_commit(bar_acc_full(acc));
+    // TMA producer (warp-uniform loop, one elected lane issues). Operand k-blocks of
+    // consecutive tiles stream through a kRing-deep ring (stage st, pass parity ph kept
+    // incrementally: no divisions on this critical path); a tile's norms go into a 4-slot
+    // ring with its first k-block. Every wait is on the completion right after the last one
+    // consumed for that barrier.
+    const uint64_t keep = policy_evict_last();
+    int st = 0;
+    uint32_t ph = 0u;
+    bool reuse = false;                                    // ring wrapped at least once
+    for (long long t = 0; t < my_tiles; ++t) {
+      int I, J;
+      tile_ij(t, I, J);
+      const int ns = (int)(t & 3);
+      if (t >= 4) mbar_wait(bar_nempty(ns), (uint32_t)(((t - 4) >> 2) & 1));        // epilogue of t-4 read slot
+      if (elect_one()) {
+        mbar_arrive_expect_tx(bar_nfull(ns), 2 * kTile * 4);
+        const uint32_t nd = sbase + Smem::NORMS + ns * 2 * kTile * 4;
+        bulk_g2s(nd, norms + I * kTile, kTile * 4, bar_nfull(ns));
+        bulk_g2s(nd + kTile * 4, norms + J * kTile, kTile * 4, bar_nfull(ns));
       }
+      __syncwarp();
+      for (int kb = 0; kb < kblocks; ++kb) {
+        if (reuse) mbar_wait(bar_free(st), ph ^ 1u);       // MMAs of the previous pass over st done
+        if (elect_one()) {
+          mbar_arrive_expect_tx(bar_full(st), (uint32_t)(2 * kStageBytes));
+          const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
+          // features stay L2-resident (evict_last) under the output stream
+          tma_load_2d_hint(ops, &tmap, kb * kKBlock, I * kTile, bar_full(st), keep);
+          tma_load_2d_hint(ops + kStageBytes, &tmap, kb * kKBlock, J * kTile, bar_full(st), keep);
+        }
+        __syncwarp();
+        if (++st == kRing) { st = 0; ph ^= 1u; reuse = true; }
+      }
+    }
+  } else if (warp == kEpiWarps + 1) {
+    // MMA issuer (warp-uniform loop, one elected lane issues): per k-block wait for its
+    // operands, four K=16 MMAs into the tile's accumulator and the commit of the stage back
+    // to the producer; per tile, commit the accumulator to the epilogue.
+    const uint64_t dbase = sw128_desc(sbase + Smem::OPS);     // + (byte offset >> 4) per operand
+    int st = 0;
+    uint32_t ph = 0u;
+    for (long long t = 0; t < my_tiles; ++t) {
+      const int acc = (int)(t & 1);
+      const uint32_t d_tmem = tmem + (uint32_t)(acc * kTile);
+      if (t >= 2) mbar_wait(bar_acc_empty(acc), (uint32_t)(((t - 2) >> 1) & 1));    // acc drained
+      for (int kb = 0; kb < kblocks; ++kb) {
+        mbar_wait(bar_full(st), ph);
+        tc_fence_after();
+        const uint64_t da = dbase + (uint64_t)((st * Smem::OPS_STAGE) >> 4);
+        if (elect_one()) tc_mma_kblock(d_tmem, da, da + (uint64_t)(kStageBytes >> 4), kIdesc, kb != 0 ? 1u : 0u, bar_free(st));
+        __syncwarp();
+        if (++st == kRing) { st = 0; ph ^= 1u; }
+      }
+      if (elect_one()) tc_commit(bar_acc_full(acc));
+      __syncwarp();
     }
   } else {
     // epilogue warps: TMEM lane quarter q, 32-column chunk cq
@@ -280,8 +331,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     const uint64_t stream_out = policy_evict_first();
     const bool storer = threadIdx.x == 0;                 // issues the tile's four TMA stores
     int it = 0;
-    for (long long t = t_beg; t < t_end; ++t, ++it) {
-      const int I = I0 + (int)(t / tiles_j), J = (int)(t % tiles_j), acc = it & 1, ns = it & 3;
+    for (long long t = 0; t < my_tiles; ++t, ++it) {
+      int I, J;
+      tile_ij(t, I, J);
+      const int acc = it & 1, ns = it & 3;
       const uint32_t nrm = snorm + ns * 2 * kTile * 4;
       mbar_wait(bar_nfull(ns), (uint32_t)((it >> 2) & 1));
       const float ni = ld_shared_f32(nrm + 4 * r);
