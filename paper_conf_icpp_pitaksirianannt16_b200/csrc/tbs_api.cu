@@ -276,9 +276,10 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
   }
   auto fill = [&](auto& op, int R, long long ka_tp) {
     op.nb = nb;
-    op.rows = LAT ? nb : nb + kGuard;
+    op.rows = nb + kGuard;
     op.inv_w = (float)(1.0 / (double)w);
     op.scale = (float)std::ldexp(1.0 / (double)m, j);
+    op.scale_up = std::nextafter((float)(std::ldexp(1.0 / (double)m, j) * (1.0 + std::ldexp(1.0, -17))), INFINITY);
     op.mj = (float)std::ldexp((double)m, -j);
     op.m = (int)m;
     op.sh = 2 * j;

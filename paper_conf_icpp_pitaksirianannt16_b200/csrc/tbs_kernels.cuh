@@ -175,6 +175,7 @@ struct SdhSmemOp {
   int rows;           // rows allocated (nb, + kGuard in float mode)
   float inv_w;        // fp32(1 / w)                       (float mode)
   float scale;        // fp32(2^j / m)                     (lattice mode)
+  float scale_up;     // fp32(2^j / m) * (1 + 2^-17), rounded up (lattice fast variant)
   int m, sh;          // w = m * 2^-j, sh = 2 j            (lattice mode)
   unsigned long long* hist;  // global u64 output [nb]
   float ymax;         // float: 2^23 + nb - 1 (clamp variant)
@@ -190,9 +191,11 @@ struct SdhSmemOp {
   __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
   // Kernel-uniform code variant, chosen once from the loader's bounding box:
   //   float mode:   0 = no clamp (every k < nb + kGuard is proven), 1 = clamp to nb-1;
-  //   lattice mode: exact fix-up in 0 = fp32 (all products < 2^24, exact in float),
-  //                 1 = 32-bit integers, 2 = 64-bit integers (general).
-  static constexpr int kVariants = LATTICE ? 3 : 2;
+  //   lattice mode: 0 = fp32 one-sided fix-up, no clamp (all products < 2^24 and every
+  //                 estimate < nb + kGuard proven; not in bucket-range passes),
+  //                 exact two-sided fix-up in 1 = fp32, 2 = 32-bit integers,
+  //                 3 = 64-bit integers (general).
+  static constexpr int kVariants = LATTICE ? 4 : 2;
   float mj;           // lattice: m * 2^-j (exact)
   __device__ __forceinline__ int variant(const uint32_t* bbox, int D) const {
     const float dmax = bbox_diameter(bbox, D);
@@ -201,10 +204,14 @@ struct SdhSmemOp {
       const double S = smax * (double)(1ull << sh);                // 4^j s_max
       const double kmax = floor(sqrt(S) / (double)m) + 2.0;         // estimate + fix-up reach
       const double e = fmax(kmax, (double)(nb + 1)) * (double)m;
-      if (smax < 8388608.0 && S < 16777216.0 && e * e < 16777216.0) return 0;
+      if (smax < 8388608.0 && S < 16777216.0 && e * e < 16777216.0) {
+        // fast variant: estimate k0 <= floor(sqrt(S) / m * (1 + 2^-16)) must stay a valid row
+        if (!RANGED && sqrt(S) / (double)m * (1.0 + 1.0 / 32768.0) + 2.0 < (double)(nb + kGuard)) return 0;
+        return 1;
+      }
       const double em = (double)(nb + 1) * (double)m;
-      if (smax < 8388608.0 && S < 4294967296.0 && em * em < 4294967296.0) return 1;
-      return 2;
+      if (smax < 8388608.0 && S < 4294967296.0 && em * em < 4294967296.0) return 2;
+      return 3;
     }
     return (dmax * inv_w < (float)(nb + kGuard - 2)) ? 0 : 1;
   }
@@ -216,7 +223,7 @@ struct SdhSmemOp {
   __device__ __forceinline__ uint32_t lattice_bucket(float s) const {
     const float q = sqrt_approx(s);
     int k = min((int)(__float_as_uint(__fmaf_rd(q, scale, kMagicF)) - kMagic), nb);
-    if (V == 2) {
+    if (V == 3) {
       const unsigned long long S = (unsigned long long)__float2uint_rz(s) << sh;
       const unsigned long long e1 = (unsigned long long)(k + 1) * (unsigned long long)m;
       k += (e1 * e1 <= S) ? 1 : 0;
@@ -272,9 +279,29 @@ struct SdhSmemOp {
         in0 = __float_as_uint(y.x) - (kMagic + (uint32_t)klo) < (uint32_t)rows;
         in1 = __float_as_uint(y.y) - (kMagic + (uint32_t)klo) < (uint32_t)rows;
       }
+    } else if (V == 0) {
+      // Lattice, fast variant. The estimate uses a scale rounded UP by 2^-17, far above the
+      // sqrt.approx + rounding error (~2^-22) and far below 1/x (x = sqrt(4^j s)/m < 4096),
+      // so k0 = floor(estimate) is k or k + 1, never less. One exact check decides:
+      //   e0 = k0 m 2^-j  (one FFMA: (2^23 + k0) mj - 2^23 mj, exact as k0 m < 2^24)
+      //   t  = s - e0^2   (one FFMA; its sign is exact: -0 never arises, t = 0 is a tie -> k0)
+      // and t < 0 (k0 = k + 1) subtracts one from bits(y) (the sign word >> 31, arithmetic,
+      // is -1) before the same LEA.HI addressing as float mode.
+      const float2 q = make_float2(sqrt_approx(s.x), sqrt_approx(s.y));
+      const float2 y = __ffma2_rd(q, make_float2(scale_up, scale_up), make_float2(kMagicF, kMagicF));
+      const float nmj = -kMagicF * mj;
+      const float2 e0 = __ffma2_rn(y, make_float2(mj, mj), make_float2(nmj, nmj));
+      const float2 t = __ffma2_rn(make_float2(-e0.x, -e0.y), e0, s);
+      constexpr int S = LOG2R + 2;
+      const uint32_t lo = (uint32_t)((threadIdx.x & (R - 1)) * 4) << (32 - S);
+      const uint32_t ub = smem_addr(tbs_smem) - (kMagic << S);
+      const uint32_t b0 = __float_as_uint(y.x) + (uint32_t)(__float_as_int(t.x) >> 31);   // bits(2^23) + k
+      const uint32_t b1 = __float_as_uint(y.y) + (uint32_t)(__float_as_int(t.y) >> 31);
+      ad0 = __funnelshift_l(lo, b0, S) + ub;
+      ad1 = __funnelshift_l(lo, b1, S) + ub;
     } else {
       uint32_t k0, k1;
-      if (V == 0) {
+      if (V == 1) {
         lattice_bucket2_f32(s, k0, k1);
       } else {
         k0 = lattice_bucket<V>(s.x);
@@ -614,6 +641,13 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
       const int cnt = min(C::TP, g.n - p0);
       const bool fast =
           (I * C::TA >= g.rb) && ((I + 1) * C::TA <= g.re) && (p0 >= (I + 1) * C::TA) && (cnt == C::TP);
+      if constexpr (Op::kVariants > 3) {
+        if (variant == 3) {
+          if (fast) run_chunk<Op, D, C, false, 3>(op, B, na, g, I, p0, cnt);
+          else run_chunk<Op, D, C, true, 3>(op, B, na, g, I, p0, cnt);
+          goto item_done;
+        }
+      }
       if constexpr (Op::kVariants > 2) {
         if (variant == 2) {
           if (fast) run_chunk<Op, D, C, false, 2>(op, B, na, g, I, p0, cnt);

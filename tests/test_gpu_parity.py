@@ -123,8 +123,9 @@ def test_sdh_degenerate(tbs, n):
 @pytest.mark.parametrize("n", [2, 17, 1500, 2048, 2049, 4096, 6001, 13824])
 def test_sdh_lattice_exact(tbs, n):
     p = g.lattice(24, 5)[:n]
-    for (w, nb) in [(1.0, 64), (0.5, 80), (0.75, 7)]:
-        m, j = (1, 0) if w == 1.0 else ((1, 1) if w == 0.5 else (3, 2))
+    # (w, nb) chosen so the bounding box selects each exact variant: the one-sided fp32
+    # fix-up without clamp (m = 1, 3, 5), the clamped two-sided fp32 fix-up (0.75, 7)
+    for (w, nb, m, j) in [(1.0, 64, 1, 0), (0.5, 80, 1, 1), (0.75, 7, 3, 2), (0.75, 80, 3, 2), (1.25, 40, 5, 2)]:
         h = sdh_gpu(tbs, p, w, nb, lattice=True)
         assert h.tolist() == oracle.sdh_lattice(p, m, j, nb).tolist(), (n, w, nb)
 
