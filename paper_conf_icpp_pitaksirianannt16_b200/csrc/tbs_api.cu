@@ -18,6 +18,7 @@
 #include "tbs.h"
 #include "tbs_kernels.cuh"
 #include "tbs_hd.cuh"
+#include "tbs_hd2.cuh"
 #include "tbs_knn.cuh"
 
 using namespace tbs;
@@ -579,8 +580,14 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
   Device dev;
   int rc = current_device(dev);
   if (rc) return rc;
+  // The CTA-pair kernel (256 x 256 tiles, half the L2 operand traffic per output, double-
+  // buffered epilogue staging; tbs_hd2.cuh) is measured faster than the one-CTA 128 x 128
+  // kernel (tbs_hd.cuh) at every d tried (64K points, d = 64: 3.10 vs 3.15 ms; d = 512:
+  // 4.60 vs 6.26 ms); TBS_HD_1SM=1 selects the one-CTA kernel (A/B runs).
+  static const bool one_sm = [] { const char* e = getenv("TBS_HD_1SM"); return e && atoi(e) != 0; }();
   const int dp = (d + hd::kKBlock - 1) / hd::kKBlock * hd::kKBlock;
-  const int64_t n_pad = (n + hd::kTile - 1) / hd::kTile * hd::kTile;
+  const int tile = one_sm ? hd::kTile : hd2::kPair;
+  const int64_t n_pad = (n + tile - 1) / tile * tile;
   unsigned char* scratch = nullptr;
   const size_t xbytes = (size_t)n_pad * dp * 2;
   TBS_CUDA(cudaMallocAsync((void**)&scratch, xbytes + (size_t)n_pad * 4, st));
@@ -623,26 +630,33 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
     }
   }
   if (!rc) {
-    const int I0 = (int)(rb / hd::kTile), I1 = (int)((re + hd::kTile - 1) / hd::kTile);
-    const int tiles_i = I1 - I0, tiles_j = (int)(n_pad / hd::kTile);
+    const int I0 = (int)(rb / tile), I1 = (int)((re + tile - 1) / tile);
+    const int tiles_i = I1 - I0, tiles_j = (int)(n_pad / tile);
     const long long ntiles = (long long)tiles_i * tiles_j;
-    const int grid = (int)std::min<long long>(ntiles, dev.sms);
-    const int smem = hd::Smem::BYTES + 1024;
+    const int grid = one_sm ? (int)std::min<long long>(ntiles, dev.sms)
+                            : 2 * (int)std::min<long long>(ntiles, dev.sms / 2);   // CTA pairs
+    const int smem = (one_sm ? hd::Smem::BYTES : hd2::Smem::BYTES) + 1024;
     const float cexp = (float)(-(double)k.gamma * 1.4426950408889634);
     const int kblocks = dp / hd::kKBlock;
     auto launch = [&](auto kern) -> int {
       TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
       if (eb) TBS_CUDA(cudaEventRecord(eb, st));
-      kern<<<grid, hd::kThreads, smem, st>>>(tmap, tmap_out, use_tma_store, norms, (int)n, kblocks, I0, tiles_i,
-                                             tiles_j, (int)rb, (int)re, cexp, out);
+      kern<<<grid, one_sm ? hd::kThreads : hd2::kThreads, smem, st>>>(tmap, tmap_out, use_tma_store, norms, (int)n,
+                                                                     kblocks, I0, tiles_i, tiles_j, (int)rb, (int)re,
+                                                                     cexp, out);
       TBS_CUDA(cudaGetLastError());
       g_launches.fetch_add(1);
       if (ee) TBS_CUDA(cudaEventRecord(ee, st));
       return TBS_OK;
     };
-    rc = k.type == 0 ? launch(hd::hd_pairmatrix_kernel<0>)
-         : k.type == 1 ? launch(hd::hd_pairmatrix_kernel<1>)
-                       : launch(hd::hd_pairmatrix_kernel<2>);
+    if (one_sm)
+      rc = k.type == 0 ? launch(hd::hd_pairmatrix_kernel<0>)
+           : k.type == 1 ? launch(hd::hd_pairmatrix_kernel<1>)
+                         : launch(hd::hd_pairmatrix_kernel<2>);
+    else
+      rc = k.type == 0 ? launch(hd2::hd_pair_kernel<0>)
+           : k.type == 1 ? launch(hd2::hd_pair_kernel<1>)
+                         : launch(hd2::hd_pair_kernel<2>);
   }
   cudaFreeAsync(scratch, st);
   return rc;
