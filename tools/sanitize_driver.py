@@ -25,6 +25,15 @@ out.append(tbs.pcf(p, 0.05).item())
 out.append(tbs.pcf(p, 0.05, rows=(7, 2000)).item())
 out.append(float(tbs.pairmatrix(p[:1001], 1.0).sum().item()))
 out.append(float(tbs.pairmatrix(p[:1000], 1.0, kernel="dist").sum().item()))
+out.append(tbs.sdh(lat, 0.75, 80, lattice=True).sum().item())     # fast lattice variant, m = 3
+out.append(tbs.sdh(lat, 0.75, 7, lattice=True).sum().item())      # clamped two-sided fp32 variant
+out.append(float(tbs.kde(p, 1.0).item()))
+out.append(float(tbs.knn(p, 8)[1].sum().item()))
+out.append(float(tbs.knn(p, 5, rows=(3, 1800))[1].sum().item()))
+xb = torch.from_numpy(g.uniform(777, 4, 96)).cuda().to(torch.bfloat16)   # hd: CTA pairs, ragged n
+out.append(float(tbs.pairmatrix_hd(xb, 0.01).sum().item()))
+out.append(float(tbs.pairmatrix_hd(xb, 0.01, rows=(130, 419)).sum().item()))
+out.append(float(tbs.pairmatrix_hd(xb[:700], 0.01, kernel="dist").sum().item()))
 big = torch.from_numpy(g.uniform(40000, 3)).cuda()                # main (non-small) tile config
 out.append(tbs.sdh(big, w, 64).sum().item())
 torch.cuda.synchronize()
