@@ -390,6 +390,42 @@ def test_pairmatrix_hd_rows_and_host(tbs):
     assert np.all(np.abs(full - ref) <= ref * (0.01 * _hd_bound(xb) + 2e-6))
 
 
+@pytest.mark.parametrize("rows", [(0, 256), (128, 384), (300, 700), (511, 513), (255, 257), (699, 700), (5, 5)])
+@pytest.mark.parametrize("n", [700, 702])
+def test_pairmatrix_hd_pair_tile_rows(tbs, rows, n):
+    """Row ranges that cut the CTA-pair tiles (256 rows: CTA 0 rows 0-127, CTA 1 rows 128-255)
+    anywhere, with n % 4 == 0 (TMA-store path) and != 0 (masked path): equal to the full matrix."""
+    import torch
+    rng = np.random.default_rng(n + rows[0])
+    xb = _bf16_bits(rng.standard_normal((n, 136)).astype(np.float32))
+    xt = torch.from_numpy(xb.view(np.int16)).cuda().view(torch.bfloat16)
+    full = tbs.pairmatrix_hd(xt, 0.01).cpu().numpy()
+    part = tbs.pairmatrix_hd(xt, 0.01, rows=rows).cpu().numpy()
+    assert part.shape == (rows[1] - rows[0], n)
+    assert np.array_equal(part, full[rows[0]:rows[1]])
+
+
+@pytest.mark.parametrize("n,d", [(9000, 64), (6000, 520)])
+def test_pairmatrix_hd_many_tiles_sampled(tbs, n, d):
+    """More pair tiles than clusters (persistent round-robin / banded raster at d > 128):
+    sampled row strips against the oracle with the derived bound."""
+    import torch
+    rng = np.random.default_rng(n + d)
+    xb = _bf16_bits(rng.random((n, d), dtype=np.float32))
+    xt = torch.from_numpy(xb.view(np.int16)).cuda().view(torch.bfloat16)
+    gamma = 1.0 / d
+    full = tbs.pairmatrix_hd(xt, gamma).cpu().numpy().astype(np.float64)
+    g32 = np.float64(np.float32(gamma))
+    for r0 in (0, 2000, n - 300):
+        rr = (r0, r0 + 300)
+        ref = oracle.pairmatrix_hd(xb, gamma, rows=rr)
+        x = (xb.astype(np.uint32) << 16).view(np.float32).astype(np.float64)
+        nrm = (x * x).sum(1)
+        ax = np.abs(x)
+        B = 2.0 ** -23 * (d / 16 + 8) * (nrm[rr[0]:rr[1], None] + nrm[None, :] + 2 * ax[rr[0]:rr[1]] @ ax.T)
+        assert np.all(np.abs(full[rr[0]:rr[1]] - ref) <= ref * (g32 * B + 2e-6) + 1e-30)
+
+
 # ------------------------------------------------------------------ NEXT-2: all-point kNN (reading R5)
 def knn_gpu(tbs, p, k, rows=None):
     import torch
