@@ -363,6 +363,15 @@ def main():
         if op in ("sdh", "sdh_lattice"):
             roof["mufu_cap"] = pk["mufu"] / 1e9         # one MUFU.SQRT per pair: this design's ceiling
             roof["frac_of_mufu_cap"] = pairs_s / pk["mufu"]
+            if nb + 32 > 768:
+                # fewer than 32 lane-private replicas fit (DESIGN.md §7 a8): the increments hit
+                # random banks of one shared copy; the measured ceiling of that access pattern
+                # (tools/peaks.cu, profiles/r01_peaks.json atoms_random_256) bounds this design
+                rp = os.path.join(ROOT, "profiles", "r01_peaks.json")
+                if os.path.exists(rp):
+                    cap = json.load(open(rp))["atoms_random_256"]["per_clk_per_sm"] * SMS * pk["f_max"]
+                    roof["atoms_random_cap"] = cap / 1e9
+                    roof["frac_of_atoms_random_cap"] = pairs_s / cap
     roof["traffic"] = None
     prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(prof):

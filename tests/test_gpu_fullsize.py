@@ -189,6 +189,40 @@ def test_pairmatrix_hd_64k_sampled_rows(tbs):
         assert np.all(np.abs(got[k] - ref) <= ref * (g32 * B + 2e-6)), r
 
 
+# ---------------------------------------------------------------- NEXT-3 at the d = 512 bench size (CTA pairs, banded raster)
+def test_pairmatrix_hd_64k_d512_sampled_rows(tbs):
+    import torch
+    n, d = 1 << 16, 512
+    x = torch.from_numpy(g.uniform(n, 7, d)).cuda().to(torch.bfloat16)
+    xb = x.view(torch.int16).cpu().numpy().view(np.uint16)
+    out = tbs.pairmatrix_hd(x, 1.0 / d)
+    rng = np.random.default_rng(2)
+    rows = sorted(set([0, 127, 128, 255, 256, n - 1] + rng.integers(0, n, 26).tolist()))
+    got = host(out.index_select(0, torch.tensor(rows, device=out.device))).astype(np.float64)
+    del out
+    torch.cuda.empty_cache()
+    xf = (xb.astype(np.uint32) << 16).view(np.float32).astype(np.float64)
+    nrm = (xf * xf).sum(1)
+    g32 = np.float64(np.float32(1.0 / d))
+    for k, r in enumerate(rows):
+        ref = oracle.pairmatrix_hd(xb, 1.0 / d, rows=(r, r + 1))[0]
+        B = 2.0 ** -23 * (d / 16 + 8) * (nrm[r] + nrm + 2 * np.abs(xf) @ np.abs(xf[r]))
+        assert np.all(np.abs(got[k] - ref) <= ref * (g32 * B + 2e-6)), r
+
+
+# ---------------------------------------------------------------- NEXT-2: kernel-density sum at the bench size
+def test_kde_1m_strips(tbs):
+    """bench.py kde_uniform_1m (N = 1M, gamma = 1): anchor strips computed through the row-range
+    API in the bench's launch configuration, each within 1e-5 relative of the oracle's strip."""
+    n = 1 << 20
+    p = g.uniform(n, 2)
+    pt = dev(p)
+    for rb, re in [(0, 300), (n // 3, n // 3 + 300), (n - 300, n)]:
+        got = float(host(tbs.kde(pt, 1.0, rows=(rb, re))))
+        ref = oracle.kde(p, 1.0, rows=(rb, re))
+        assert abs(got - ref) <= 1e-5 * ref, (rb, got, ref)
+
+
 # ---------------------------------------------------------------- NEXT-2: kNN at the bench size
 def test_knn_1m_sampled_strips(tbs):
     """bench.py knn_uniform_1m_k8: 1M uniform points, k = 8 (3 partner segments + merge)."""
