@@ -638,12 +638,24 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
     const int smem = (one_sm ? hd::Smem::BYTES : hd2::Smem::BYTES) + 1024;
     const float cexp = (float)(-(double)k.gamma * 1.4426950408889634);
     const int kblocks = dp / hd::kKBlock;
+    // CTA-pair tile raster: bands of `band` tile rows walked column by column, tiles dealt
+    // round-robin over clusters (0: contiguous row-major range per cluster). TBS_HD_BAND overrides.
+    static const int band_env = [] { const char* e = getenv("TBS_HD_BAND"); return e ? atoi(e) : -1; }();
+    // Default: contiguous ranges for d <= 128 (output-bound; banding measured 3.19 vs 3.08 ms
+    // at 64K x 64), else bands whose A rows hold ~8 MiB of features (64K x 512: band 32;
+    // measured 8: 4.56, 16: 4.45, 32: 4.12, 64: 4.11, 128: 4.57, 256: 4.90 ms).
+    const int band = band_env >= 0 ? band_env
+                     : kblocks <= 2 ? 0
+                                    : (int)std::max<long long>(1, (8ll << 20) / ((long long)hd2::kPair * dp * 2));
     auto launch = [&](auto kern) -> int {
       TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
       if (eb) TBS_CUDA(cudaEventRecord(eb, st));
-      kern<<<grid, one_sm ? hd::kThreads : hd2::kThreads, smem, st>>>(tmap, tmap_out, use_tma_store, norms, (int)n,
-                                                                     kblocks, I0, tiles_i, tiles_j, (int)rb, (int)re,
-                                                                     cexp, out);
+      if constexpr (std::is_same<decltype(kern), decltype(&hd2::hd_pair_kernel<0>)>::value)
+        kern<<<grid, hd2::kThreads, smem, st>>>(tmap, tmap_out, use_tma_store, norms, (int)n, kblocks, I0, tiles_i,
+                                                tiles_j, (int)rb, (int)re, cexp, out, band);
+      else
+        kern<<<grid, hd::kThreads, smem, st>>>(tmap, tmap_out, use_tma_store, norms, (int)n, kblocks, I0, tiles_i,
+                                               tiles_j, (int)rb, (int)re, cexp, out);
       TBS_CUDA(cudaGetLastError());
       g_launches.fetch_add(1);
       if (ee) TBS_CUDA(cudaEventRecord(ee, st));

@@ -31,7 +31,6 @@ constexpr int kHalf = 128;                         // rows (and B rows) per CTA
 constexpr int kRing = 4;                           // operand ring: 4 x (A 16 KB | B 16 KB) per CTA
 constexpr int kThreads = (kEpiWarps + 2) * 32;     // + a TMA producer warp and an MMA warp
 constexpr int kTmemCols = 512;                     // two 256-column fp32 accumulators
-constexpr int kBand = 8;                           // pair-tile rows per raster band
 constexpr int kNorms = kHalf + kPair;              // per slot: 128 row norms | 256 column norms
 constexpr uint32_t kPeerMask = 0xFEFFFFFFu;        // clears the CTA-rank bit of a shared::cluster address
 constexpr int kQuarter = 64;                       // columns per epilogue staging step
@@ -123,7 +122,7 @@ template <int KTYPE>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     hd_pair_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ CUtensorMap tmap_out,
                    int use_tma_store, const float* __restrict__ norms, int n, int kblocks, int I0, int tiles_i,
-                   int tiles_j, int rb, int re, float cexp, float* __restrict__ out) {
+                   int tiles_j, int rb, int re, float cexp, float* __restrict__ out, int band) {
   extern __shared__ __align__(1024) unsigned char hd2_smem_raw[];
   unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(hd2_smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sbase = smem_addr(sm);
@@ -142,9 +141,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   const int cid = (int)(blockIdx.x >> 1), nclusters = (int)(gridDim.x >> 1);
   const long long ntiles = (long long)tiles_i * tiles_j;
 
-  // Pair tiles: banded round-robin raster for operand-heavy shapes, contiguous row-major
-  // ranges for output-bound shapes (see tbs_hd.cuh); both CTAs of a pair walk the same list.
-  const bool banded = kblocks > 2;
+  // Pair tiles: round-robin over clusters in bands of `band` tile rows walked column by column
+  // (operand-heavy shapes: the tiles in flight share A bands and B columns in L2), or
+  // contiguous row-major ranges (band = 0); both CTAs of a pair walk the same list.
+  const bool banded = band > 0;
   const long long c_beg = ntiles * cid / nclusters;
   const long long my_tiles = banded ? (ntiles > cid ? (ntiles - 1 - cid) / nclusters + 1 : 0)
                                     : ntiles * (cid + 1) / nclusters - c_beg;
@@ -156,10 +156,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       return;
     }
     const long long t = (long long)cid + k * nclusters;
-    const long long band = t / ((long long)kBand * tiles_j);
-    const long long w = t - band * kBand * tiles_j;
-    const int rows = min(kBand, tiles_i - (int)band * kBand);
-    I = I0 + (int)band * kBand + (int)(w % rows);
+    const long long bi = t / ((long long)band * tiles_j);
+    const long long w = t - bi * band * tiles_j;
+    const int rows = min(band, tiles_i - (int)bi * band);
+    I = I0 + (int)bi * band + (int)(w % rows);
     J = (int)(w / rows);
   };
 
