@@ -52,12 +52,25 @@ using namespace tbs;
 #ifndef TBS_LAT_MINB
 #define TBS_LAT_MINB 2
 #endif
+// Lattice fast variant (fp32 one-sided fix-up) compiled on its own: smaller register
+// footprint than the kernel holding every exact-bucketing variant.
+#ifndef TBS_LATF_KA
+#define TBS_LATF_KA 8
+#endif
+#ifndef TBS_LATF_TP
+#define TBS_LATF_TP 1024
+#endif
+#ifndef TBS_LATF_MINB
+#define TBS_LATF_MINB 3
+#endif
+#define TBS_LATF_CFG TBS_LATF_KA, TBS_LATF_TP, TBS_LATF_MINB
 #define TBS_SDH_CFG TBS_SDH_KA, TBS_SDH_TP, TBS_SDH_MINB
 #define TBS_PCF_CFG TBS_PCF_KA, TBS_PCF_TP, TBS_PCF_MINB
 #define TBS_LAT_CFG TBS_LAT_KA, TBS_LAT_TP, TBS_LAT_MINB
 using SdhCfg = Cfg<TBS_SDH_CFG>;
 using PcfCfg = Cfg<TBS_PCF_CFG>;
 using LatCfg = Cfg<TBS_LAT_CFG>;
+using LatFastCfg = Cfg<TBS_LATF_CFG>;
 // Small problems (fewer work items than ~2 per SM with the main configs): finer tiles so
 // the grid covers the GPU (BASELINE configs[0], N = 4096, is launch/latency-bound).
 #ifndef TBS_SMALL_TP
@@ -140,12 +153,12 @@ int pad_rows(int64_t n) { return (int)(((n + kPadAlign - 1) / kPadAlign) * kPadA
 int D_of(const tbs_args* a) { return a->dim <= 3 ? 3 : 4; }
 
 // Persistent grid for a pair-kernel instantiation: SMs x resident CTAs (at most one CTA per item).
-template <class Op, int D, class C>
+template <class Op, int D, class C, int VSET = 0x1F>
 int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op& op, const uint32_t* bbox,
                 cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee, bool first_launch_on_scratch = true) {
   // bbox may be nulled (TBS_FORCE_CLAMP); the 64-byte block always follows the SoA copy
   const uint32_t* bbox_block = reinterpret_cast<const uint32_t*>(soa + (size_t)D_of(a) * pad_rows(a->n));
-  auto kern = pair_kernel<Op, D, C>;
+  auto kern = pair_kernel<Op, D, C, VSET>;
   Geom g = make_geom(a->n, a->row_begin, a->row_end, C::TA, C::TP);
   // work queue head: the last u64 of the 64-byte bounding-box block (zeroed by the call's
   // memset; re-zeroed here for every further launch on the same scratch, e.g. bucket passes)
@@ -255,6 +268,21 @@ struct SdhPlan {
   int pass_rows = 0;    // buckets per pass
 };
 
+// Lattice mode: the fast variants 4 and 0 (their own instantiation, LatFastCfg) and the
+// exact general variants 1-3 (LatCfg) are two launches; the one whose variant the bounding box does
+// not select exits at once (the work-queue counter is untouched by it).
+template <class Op, int D, class C, bool LAT>
+int launch_sdh(const Device& dev, const float* soa, const tbs_args* g, const Op& op, const uint32_t* bbox,
+               cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee) {
+  if constexpr (!LAT) {
+    return launch_pair<Op, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+  } else {
+    int rc = launch_pair<Op, D, LatFastCfg, 0x11>(dev, soa, g, op, bbox, st, eb, nullptr);
+    if (rc) return rc;
+    return launch_pair<Op, D, C, 0xE>(dev, soa, g, op, bbox, st, nullptr, ee);
+  }
+}
+
 template <int D, bool LAT>
 int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const uint32_t* bbox, const tbs_args* g, float w,
                  long long m, int j, int nb, unsigned long long* hist, unsigned long long* part, int G, cudaStream_t st,
@@ -281,11 +309,13 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
     op.inv_w = (float)(1.0 / (double)w);
     op.scale = (float)std::ldexp(1.0 / (double)m, j);
     op.scale_up = std::nextafter((float)(std::ldexp(1.0 / (double)m, j) * (1.0 + std::ldexp(1.0, -17))), INFINITY);
+    op.scale_b = std::nextafter((float)(std::ldexp(1.0 / (double)m, j) * (1.0 + std::ldexp(1.0, -19))), INFINITY);
     op.mj = (float)std::ldexp((double)m, -j);
     op.m = (int)m;
     op.sh = 2 * j;
     op.hist = hist;
     // per item, a replica receives at most (32/R) lanes x kWarps x KA x TP increments
+    if (LAT) ka_tp = std::max<long long>(ka_tp, (long long)LatFastCfg::KA * LatFastCfg::TP);
     const long long per_item = (long long)(32 / R) * kWarps * ka_tp;
     op.flush_every = (int)std::max<long long>(1, (0xffffffffll / per_item) - 1);
   };
@@ -308,37 +338,39 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
   switch (pl.log2r) {
     case 5: {
       SdhSmemOp<5, LAT> op{};
-      if (small) {
-        fill(op, 32, (long long)SmallCfg::KA * SmallCfg::TP);
-        return launch_pair<SdhSmemOp<5, LAT>, D, SmallCfg>(dev, soa, g, op, bbox, st, eb, ee);
+      if constexpr (!LAT) {   // (lattice mode never takes the small-problem config)
+        if (small) {
+          fill(op, 32, (long long)SmallCfg::KA * SmallCfg::TP);
+          return launch_pair<SdhSmemOp<5, LAT>, D, SmallCfg>(dev, soa, g, op, bbox, st, eb, ee);
+        }
       }
       fill(op, 32, (long long)C::KA * C::TP);
-      return launch_pair<SdhSmemOp<5, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<5, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
     }
     case 4: {
       SdhSmemOp<4, LAT> op{};
       fill(op, 16, (long long)C::KA * C::TP);
-      return launch_pair<SdhSmemOp<4, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<4, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
     }
     case 3: {
       SdhSmemOp<3, LAT> op{};
       fill(op, 8, (long long)C::KA * C::TP);
-      return launch_pair<SdhSmemOp<3, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<3, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
     }
     case 2: {
       SdhSmemOp<2, LAT> op{};
       fill(op, 4, (long long)C::KA * C::TP);
-      return launch_pair<SdhSmemOp<2, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<2, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
     }
     case 1: {
       SdhSmemOp<1, LAT> op{};
       fill(op, 2, (long long)C::KA * C::TP);
-      return launch_pair<SdhSmemOp<1, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<1, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
     }
     default: {
       SdhSmemOp<0, LAT> op{};
       fill(op, 1, (long long)C::KA * C::TP);
-      return launch_pair<SdhSmemOp<0, LAT>, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<0, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
     }
   }
 }

@@ -176,6 +176,7 @@ struct SdhSmemOp {
   float inv_w;        // fp32(1 / w)                       (float mode)
   float scale;        // fp32(2^j / m)                     (lattice mode)
   float scale_up;     // fp32(2^j / m) * (1 + 2^-17), rounded up (lattice fast variant)
+  float scale_b;      // fp32(2^j / m) * (1 + 2^-19), rounded up (lattice bias-only variant)
   int m, sh;          // w = m * 2^-j, sh = 2 j            (lattice mode)
   unsigned long long* hist;  // global u64 output [nb]
   float ymax;         // float: 2^23 + nb - 1 (clamp variant)
@@ -191,11 +192,13 @@ struct SdhSmemOp {
   __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
   // Kernel-uniform code variant, chosen once from the loader's bounding box:
   //   float mode:   0 = no clamp (every k < nb + kGuard is proven), 1 = clamp to nb-1;
-  //   lattice mode: 0 = fp32 one-sided fix-up, no clamp (all products < 2^24 and every
+  //   lattice mode: 4 = bias only, no fix-up and no clamp (see below; every bucket edge
+  //                 the data can reach is far enough from the estimate's error),
+  //                 0 = fp32 one-sided fix-up, no clamp (all products < 2^24 and every
   //                 estimate < nb + kGuard proven; not in bucket-range passes),
   //                 exact two-sided fix-up in 1 = fp32, 2 = 32-bit integers,
   //                 3 = 64-bit integers (general).
-  static constexpr int kVariants = LATTICE ? 4 : 2;
+  static constexpr int kVariants = LATTICE ? 5 : 2;
   float mj;           // lattice: m * 2^-j (exact)
   __device__ __forceinline__ int variant(const uint32_t* bbox, int D) const {
     const float dmax = bbox_diameter(bbox, D);
@@ -204,6 +207,16 @@ struct SdhSmemOp {
       const double S = smax * (double)(1ull << sh);                // 4^j s_max
       const double kmax = floor(sqrt(S) / (double)m) + 2.0;         // estimate + fix-up reach
       const double e = fmax(kmax, (double)(nb + 1)) * (double)m;
+      // Bias-only variant: x = sqrt(4^j s) / m, k = floor(x). The estimate q c with
+      // q = sqrt.approx(s) (|rel err| <= 2^-22, measured exhaustively over every integer
+      // s < 2^24: tools/sqrt_bound.cu) and c = 2^j/m (1 + 2^-19) rounded up lies in
+      // [x, x (1 + g)], g < 2^-18. Below the next edge, S = 4^j s <= X^2 - 1 with X = (k+1) m
+      // (integers), so x <= (k+1)(1 - 1/(2 X^2)): floor(q c) = k whenever 2 X^2 g < 1,
+      // i.e. X^2 < 2^17 for the largest X the bounding box allows.
+      const double xmax = sqrt(S) / (double)m;
+      const double X = (floor(xmax) + 1.0) * (double)m;
+      if (!RANGED && smax < 16777216.0 && X * X < 131072.0 && xmax * (1.0 + 1.0 / 262144.0) + 2.0 < (double)(nb + kGuard))
+        return 4;
       if (smax < 8388608.0 && S < 16777216.0 && e * e < 16777216.0) {
         // fast variant: estimate k0 <= floor(sqrt(S) / m * (1 + 2^-16)) must stay a valid row
         if (!RANGED && sqrt(S) / (double)m * (1.0 + 1.0 / 32768.0) + 2.0 < (double)(nb + kGuard)) return 0;
@@ -259,10 +272,12 @@ struct SdhSmemOp {
   __device__ __forceinline__ void pair2(float2 s, int pv, int a0, int a1) {
     uint32_t ad0, ad1;
     bool in0 = true, in1 = true;
-    if (!LATTICE) {
+    if (!LATTICE || V == 4) {
+      // float mode, or the lattice bias-only variant (estimate scale c instead of 1/w)
+      const float c = LATTICE ? scale_b : inv_w;
       const float2 q = make_float2(sqrt_approx(s.x), sqrt_approx(s.y));
-      float2 y = __ffma2_rd(q, make_float2(inv_w, inv_w), make_float2(kMagicF, kMagicF));
-      if (V == 1) {
+      float2 y = __ffma2_rd(q, make_float2(c, c), make_float2(kMagicF, kMagicF));
+      if (!LATTICE && V == 1) {
         y.x = fminf(y.x, ymax);
         y.y = fminf(y.y, ymax);
       }
@@ -559,7 +574,10 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
   }
 }
 
-template <class Op, int D, class C>
+// VSET: bit v set = code variant v is compiled into this instantiation. A launch whose
+// kernel-uniform variant is not in VSET exits at once, so a variant with a smaller register
+// footprint can be compiled (and made resident) on its own and launched beside the rest.
+template <class Op, int D, class C, int VSET = 0x1F>
 __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __restrict__ soa, Geom g, Op op,
                                                             const uint32_t* __restrict__ bbox) {
   unsigned char* smem = tbs_smem;
@@ -573,6 +591,7 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
   if (g.trace != nullptr && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
   op.init(smem);
   const int variant = op.variant(bbox, D);
+  if (!((VSET >> variant) & 1)) return;   // CTA-uniform: another launch owns this variant
   if (tid == 0) {
     mbar_init(bar0, 1);
     mbar_init(bar1, 1);
@@ -641,29 +660,38 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
       const int cnt = min(C::TP, g.n - p0);
       const bool fast =
           (I * C::TA >= g.rb) && ((I + 1) * C::TA <= g.re) && (p0 >= (I + 1) * C::TA) && (cnt == C::TP);
-      if constexpr (Op::kVariants > 3) {
+      if constexpr (Op::kVariants > 4 && (VSET & 16)) {
+        if (variant == 4) {
+          if (fast) run_chunk<Op, D, C, false, 4>(op, B, na, g, I, p0, cnt);
+          else run_chunk<Op, D, C, true, 4>(op, B, na, g, I, p0, cnt);
+          goto item_done;
+        }
+      }
+      if constexpr (Op::kVariants > 3 && (VSET & 8)) {
         if (variant == 3) {
           if (fast) run_chunk<Op, D, C, false, 3>(op, B, na, g, I, p0, cnt);
           else run_chunk<Op, D, C, true, 3>(op, B, na, g, I, p0, cnt);
           goto item_done;
         }
       }
-      if constexpr (Op::kVariants > 2) {
+      if constexpr (Op::kVariants > 2 && (VSET & 4)) {
         if (variant == 2) {
           if (fast) run_chunk<Op, D, C, false, 2>(op, B, na, g, I, p0, cnt);
           else run_chunk<Op, D, C, true, 2>(op, B, na, g, I, p0, cnt);
           goto item_done;
         }
       }
-      if constexpr (Op::kVariants > 1) {
+      if constexpr (Op::kVariants > 1 && (VSET & 2)) {
         if (variant == 1) {
           if (fast) run_chunk<Op, D, C, false, 1>(op, B, na, g, I, p0, cnt);
           else run_chunk<Op, D, C, true, 1>(op, B, na, g, I, p0, cnt);
           goto item_done;
         }
       }
-      if (fast) run_chunk<Op, D, C, false, 0>(op, B, na, g, I, p0, cnt);
-      else run_chunk<Op, D, C, true, 0>(op, B, na, g, I, p0, cnt);
+      if constexpr (VSET & 1) {
+        if (fast) run_chunk<Op, D, C, false, 0>(op, B, na, g, I, p0, cnt);
+        else run_chunk<Op, D, C, true, 0>(op, B, na, g, I, p0, cnt);
+      }
       goto item_done;  // (keeps the label referenced for single-variant ops)
     item_done:
       __syncthreads();

@@ -123,11 +123,40 @@ def test_sdh_degenerate(tbs, n):
 @pytest.mark.parametrize("n", [2, 17, 1500, 2048, 2049, 4096, 6001, 13824])
 def test_sdh_lattice_exact(tbs, n):
     p = g.lattice(24, 5)[:n]
-    # (w, nb) chosen so the bounding box selects each exact variant: the one-sided fp32
-    # fix-up without clamp (m = 1, 3, 5), the clamped two-sided fp32 fix-up (0.75, 7)
-    for (w, nb, m, j) in [(1.0, 64, 1, 0), (0.5, 80, 1, 1), (0.75, 7, 3, 2), (0.75, 80, 3, 2), (1.25, 40, 5, 2)]:
+    # (w, nb) chosen so the bounding box selects each exact variant (d_max = 23 sqrt(3)):
+    # bias only, X = (k_max + 1) m < 362 (w = 1, 1/2, 3/4 @ 80, 5/4, 1/8 with X = 319), the
+    # one-sided fp32 fix-up without clamp (1/16: X = 638; 3/32: X = 1275), the clamped
+    # two-sided fp32 fix-up (3/4 @ 7 buckets)
+    for (w, nb, m, j) in [(1.0, 64, 1, 0), (0.5, 80, 1, 1), (0.75, 7, 3, 2), (0.75, 80, 3, 2), (1.25, 40, 5, 2),
+                          (0.125, 320, 1, 3), (0.0625, 640, 1, 4), (0.09375, 400, 3, 5)]:
         h = sdh_gpu(tbs, p, w, nb, lattice=True)
         assert h.tolist() == oracle.sdh_lattice(p, m, j, nb).tolist(), (n, w, nb)
+
+
+def test_sdh_lattice_bias_only_boundary(tbs):
+    """Bias-only exact variant at its limit: lattice {0..208}^3, w = 1, so the largest
+    X = (k_max + 1) m = 361 (361^2 = 130321 < 2^17); every s = k^2 + 2k (one below the next
+    edge) and every exact square k^2 up to 360^2 that the subset reaches must bucket exactly."""
+    p = g.lattice(209, 21)[:15000]
+    p = np.concatenate([p, np.array([[0, 0, 0], [208, 208, 208], [208, 0, 0], [0, 208, 208]], np.float32)])
+    h = sdh_gpu(tbs, p, 1.0, 400, lattice=True)
+    assert h.tolist() == oracle.sdh_lattice(p, 1, 0, 400).tolist()
+
+
+def test_sqrt_approx_bound():
+    """The bias-only lattice variant assumes |sqrt.approx(s) / sqrt(s) - 1| <= 2^-22 for every
+    integer s < 2^24 (exhaustive on this GPU; tools/sqrt_bound.cu), with its 2^-19 bias
+    leaving a 4x margin."""
+    import json
+    import os
+    import subprocess
+    import tempfile
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    exe = os.path.join(tempfile.mkdtemp(), "sqrt_bound")
+    subprocess.run([os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc"), "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-o", exe,
+                    os.path.join(root, "tools", "sqrt_bound.cu")], check=True)
+    r = json.loads(subprocess.run([exe], check=True, capture_output=True, text=True).stdout)
+    assert r["log2_int"] <= -22.0 and r["log2_1_4"] <= -22.0, r
 
 
 @pytest.mark.parametrize("mode", [None, "lane", "cta", "global"])

@@ -1,0 +1,40 @@
+// Exhaustive relative-error bound of sqrt.approx.ftz.f32 on sm_100a, the assumption behind
+// the bias-only exact lattice variant (lattice mode): every integer s in
+// [1, 2^24) (the whole lattice-mode domain of squared distances) and every fp32 in [1, 4)
+// (one full period of the exponent parity). Prints one JSON line.
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o sqrt_bound tools/sqrt_bound.cu
+#include <cstdio>
+#include <cstdint>
+#include <cmath>
+#include <cstring>
+#include <cuda_runtime.h>
+
+__device__ unsigned long long g_max[2];   // max relative error as ordered double bits
+
+__global__ void k_bound(int mode, uint32_t count) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= count) return;
+  // mode 0: integers 1 .. 2^24-1; mode 1: fp32 in [1, 4) (bits 0x3f800000 .. 0x407fffff)
+  const float x = mode == 0 ? (float)(i + 1) : __uint_as_float(0x3f800000u + i);
+  float q;
+  asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(q) : "f"(x));
+  const double t = sqrt((double)x);
+  const double e = fabs((double)q - t) / t;
+  atomicMax(&g_max[mode], (unsigned long long)__double_as_longlong(e));   // e >= 0: bits are ordered
+}
+
+int main() {
+  const uint32_t n0 = (1u << 24) - 1, n1 = 0x407fffffu - 0x3f800000u + 1;
+  unsigned long long z[2] = {0, 0}, h[2];
+  if (cudaMemcpyToSymbol(g_max, z, sizeof(z)) != cudaSuccess) return 1;
+  k_bound<<<(n0 + 255) / 256, 256>>>(0, n0);
+  k_bound<<<(n1 + 255) / 256, 256>>>(1, n1);
+  if (cudaDeviceSynchronize() != cudaSuccess) return 1;
+  cudaMemcpyFromSymbol(h, g_max, sizeof(h));
+  double e0, e1;
+  memcpy(&e0, &h[0], 8);
+  memcpy(&e1, &h[1], 8);
+  printf("{\"max_rel_err_int\": %.6e, \"log2_int\": %.3f, \"max_rel_err_1_4\": %.6e, \"log2_1_4\": %.3f}\n", e0,
+         log2(e0), e1, log2(e1));
+  return 0;
+}
