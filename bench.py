@@ -256,13 +256,27 @@ def main():
         rows_pm = (n * rank // world, n * (rank + 1) // world)
         out = torch.empty((rows_pm[1] - rows_pm[0], n), dtype=torch.float32, device=dev)
 
+    # N > 1, Type-I/II: the combine is fused into the kernels' flush (every partial is added
+    # into every rank's buffer over NVLink peer memory, TBS_OUT_PEERS); NCCL all_reduce only
+    # if the peer mapping cannot be set up.
+    sink, combine = None, "none"
+    if pg is not None and op in ("sdh", "sdh_lattice", "pcf"):
+        try:
+            sink = tbs.PeerSink(nb if op != "pcf" else 1, pg, dev)
+            combine = "fused-peer"
+        except Exception as e:   # noqa: BLE001 — report and use the collective instead
+            print(f"[bench] fused combine unavailable ({e}); using NCCL all_reduce", file=sys.stderr)
+            combine = "nccl-allreduce"
+    elif pg is not None:
+        combine = "nccl-allreduce" if op == "kde" else "none (row-sharded output)"
+
     def step(events=None):
         if op == "sdh":
-            tbs.sdh(pts, w, nb, out=out, events=events, group=pg)
+            tbs.sdh(pts, w, nb, out=out, events=events, group=pg, sink=sink)
         elif op == "sdh_lattice":
-            tbs.sdh(pts, w, nb, lattice=True, out=out, events=events, group=pg)
+            tbs.sdh(pts, w, nb, lattice=True, out=out, events=events, group=pg, sink=sink)
         elif op == "pcf":
-            tbs.pcf(pts, params["r"], out=out, events=events, group=pg)
+            tbs.pcf(pts, params["r"], out=out, events=events, group=pg, sink=sink)
         elif op == "kde":
             tbs.kde(pts, params["gamma"], out=out, events=events, group=pg)
         elif op == "pairmatrix_hd":
@@ -404,13 +418,13 @@ def main():
             def e2e_step():
                 d = ph.to(dev, non_blocking=True)
                 if op == "sdh":
-                    r = tbs.sdh(d, w, nb, group=pg)
+                    r = tbs.sdh(d, w, nb, group=pg, sink=sink)
                 elif op == "kde":
                     r = tbs.kde(d, params["gamma"], group=pg)
                 elif op == "knn":
                     r = tbs.knn(d, params["k"], group=pg)[1]
                 else:
-                    r = tbs.pcf(d, params["r"], group=pg)
+                    r = tbs.pcf(d, params["r"], group=pg, sink=sink)
                 res_h.copy_(r)
         for _ in range(2):
             e2e_step()
@@ -440,7 +454,8 @@ def main():
                "l2": "flushed between steps (256 MiB write between the per-step CUDA events; inputs 12 B/point < L2)",
                "timed_region_ms": region_ms,
                "parallelism": f"rows{world}" if world > 1 else "single",
-               "step": "loader + pair kernel + flush" + (" + all_reduce" if world > 1 and op != "pairmatrix" else "")}
+               "step": "loader + pair kernel + flush" + (f" + combine ({combine})" if world > 1 else ""),
+               "combine": combine}
         if op == "sdh":
             cfg["bucket_width"] = w
         line = {"metric": METRIC if op in ("sdh", "sdh_lattice") else f"{op} throughput ({unit})",
@@ -450,6 +465,8 @@ def main():
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
                 "clocks": ck}
         print(json.dumps(line), flush=True)
+    if sink is not None:
+        sink.close()
     if pg is not None:
         dist.destroy_process_group()
 

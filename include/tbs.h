@@ -79,6 +79,15 @@ typedef struct {
 #define TBS_HIST_FORCE_GLOBAL 0x40u   /* SDH: partially privatised global u64 copies       */
 #define TBS_FORCE_CLAMP 0x100u        /* SDH: never elide the nb-1 clamp (ablation/tests)   */
 #define TBS_HIST_FORCE_PASSES 0x200u  /* SDH: bucket-range passes with one smem copy (tests)   */
+/* SDH / 2PCF: fused multi-GPU combine (the paper's multi-GPU future work,
+ * L1254-1256). Instead of writing hist / count, every partial the kernels flush (a9) is added
+ * with a system-scope atomic into EACH of args->out_peers[0 .. n_out_peers) — uint64 [nb]
+ * (SDH) or [1] (2PCF) device buffers, the local rank's own and the other ranks' mapped over
+ * NVLink by CUDA IPC (tbs_peer_open). Nothing is zeroed: the caller zeroes every rank's buffer
+ * before any rank's call starts, and after every rank's call has completed each buffer holds
+ * the sum over all ranks' row ranges (the all-reduce, without a separate collective).
+ * hist / count may be NULL. Other entry points return TBS_EUNSUPPORTED for this flag. */
+#define TBS_OUT_PEERS 0x400u
 
 #define TBS_MAX_N ((int64_t)1 << 30)
 #define TBS_MAX_BUCKETS (1 << 24)
@@ -105,7 +114,10 @@ typedef struct {
   uint32_t flags;       /* TBS_* flags above                                               */
   void* ev_begin;       /* optional cudaEvent_t recorded just before the pair kernel        */
   void* ev_end;         /* optional cudaEvent_t recorded just after it (profiling hook)     */
+  void* const* out_peers; /* TBS_OUT_PEERS: device pointers of every rank's output buffer     */
+  int n_out_peers;      /* 1 .. TBS_MAX_PEERS                                              */
 } tbs_args;
+#define TBS_MAX_PEERS 16
 
 int tbs_sdh_ex(const tbs_args* args, float bucket_width, int nbuckets, uint64_t* hist);
 int tbs_pcf_ex(const tbs_args* args, float radius, uint64_t* count);
@@ -155,6 +167,16 @@ int tbs_pairmatrix_hd_ex(const uint16_t* features, int64_t n, int d, int64_t row
  * `world` gets [*row_begin, *row_end) such that sum over its rows of (n-1-i) is
  * n(n-1)/(2*world) up to one row; the ranges are disjoint and cover [0, n). Host-only. */
 int tbs_rank_rows(int64_t n, int world, int rank, int64_t* row_begin, int64_t* row_end);
+
+/* Plumbing of the fused combine (host-only, CUDA IPC; TBS_OUT_PEERS). tbs_peer_alloc makes a
+ * zeroed device buffer of `bytes` on the current device (its own cudaMalloc allocation, so
+ * the IPC mapping starts at offset 0) and writes its 64-byte IPC handle to `handle`;
+ * tbs_peer_open maps another process's buffer from its handle (peer access over NVLink is
+ * enabled by the mapping); tbs_peer_close unmaps; tbs_peer_free frees an own buffer. */
+int tbs_peer_alloc(uint64_t bytes, void** dev_ptr, void* handle);
+int tbs_peer_open(const void* handle, void** dev_ptr);
+int tbs_peer_close(void* dev_ptr);
+int tbs_peer_free(void* dev_ptr);
 
 /* Thread-local text of the last non-OK status ("" if none). */
 const char* tbs_last_error(void);

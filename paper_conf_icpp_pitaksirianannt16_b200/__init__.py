@@ -33,6 +33,8 @@ TBS_HIST_FORCE_CTA = 0x20
 TBS_HIST_FORCE_GLOBAL = 0x40
 TBS_FORCE_CLAMP = 0x100
 TBS_HIST_FORCE_PASSES = 0x200
+TBS_OUT_PEERS = 0x400
+TBS_MAX_PEERS = 16
 KERNELS = {"gaussian": 0, "dist2": 1, "dist": 2}
 HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "global": TBS_HIST_FORCE_GLOBAL,
               "passes": TBS_HIST_FORCE_PASSES}
@@ -40,7 +42,8 @@ HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "
 # Symbols declared in include/tbs.h (checked by tests/test_abi.py).
 EXPORTS = ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
            "tbs_kde", "tbs_kde_ex", "tbs_knn", "tbs_knn_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex",
-           "tbs_rank_rows", "tbs_last_error", "tbs_release", "tbs_launch_count", "tbs_version")
+           "tbs_rank_rows", "tbs_peer_alloc", "tbs_peer_open", "tbs_peer_close", "tbs_peer_free",
+           "tbs_last_error", "tbs_release", "tbs_launch_count", "tbs_version")
 
 
 class TbsError(RuntimeError):
@@ -50,7 +53,8 @@ class TbsError(RuntimeError):
 class _Args(ctypes.Structure):
     _fields_ = [("points", ctypes.c_void_p), ("n", ctypes.c_int64), ("dim", ctypes.c_int),
                 ("row_begin", ctypes.c_int64), ("row_end", ctypes.c_int64), ("stream", ctypes.c_void_p),
-                ("flags", ctypes.c_uint32), ("ev_begin", ctypes.c_void_p), ("ev_end", ctypes.c_void_p)]
+                ("flags", ctypes.c_uint32), ("ev_begin", ctypes.c_void_p), ("ev_end", ctypes.c_void_p),
+                ("out_peers", ctypes.POINTER(ctypes.c_void_p)), ("n_out_peers", ctypes.c_int)]
 
 
 class _Kernel(ctypes.Structure):
@@ -83,11 +87,16 @@ def lib() -> ctypes.CDLL:
         L.tbs_pairmatrix_hd_ex.argtypes = [vp, i64, ctypes.c_int, i64, i64, _Kernel, vp, vp, vp, vp]
         L.tbs_rank_rows.argtypes = [i64, ctypes.c_int, ctypes.c_int, ctypes.POINTER(ctypes.c_int64),
                                     ctypes.POINTER(ctypes.c_int64)]
+        L.tbs_peer_alloc.argtypes = [ctypes.c_uint64, ctypes.POINTER(ctypes.c_void_p), ctypes.c_char_p]
+        L.tbs_peer_open.argtypes = [ctypes.c_char_p, ctypes.POINTER(ctypes.c_void_p)]
+        L.tbs_peer_close.argtypes = [vp]
+        L.tbs_peer_free.argtypes = [vp]
         L.tbs_last_error.restype = ctypes.c_char_p
         L.tbs_launch_count.restype = ctypes.c_uint64
         L.tbs_release.restype = None
         for f in ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
-                  "tbs_kde", "tbs_kde_ex", "tbs_knn", "tbs_knn_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex", "tbs_rank_rows", "tbs_version"):
+                  "tbs_kde", "tbs_kde_ex", "tbs_knn", "tbs_knn_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex", "tbs_rank_rows", "tbs_version",
+                  "tbs_peer_alloc", "tbs_peer_open", "tbs_peer_close", "tbs_peer_free"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -131,6 +140,93 @@ def partition(n: int, group=None, rows=None):
     return rank_rows(n, dist.get_world_size(group), dist.get_rank(group))
 
 
+class PeerSink:
+    """Buffers of the fused combine (TBS_OUT_PEERS): one int64[words] device buffer per rank
+    of `group`, each mapped into every rank (CUDA IPC; over NVLink between GPUs). A call
+    with ``sink=`` adds every partial its kernels flush into all of them, so after
+    ``finish()`` each rank's buffer holds the all-reduced result — the collective is fused
+    into the kernels' flush instead of a separate NCCL all_reduce.
+
+    Protocol per result: ``begin(stream)`` zeroes this rank's buffer and waits (stream sync +
+    barrier) until every rank has zeroed; the compute call adds; ``finish(stream)`` waits
+    (stream sync + barrier) until every rank's kernels have completed and returns a copy of
+    the local buffer."""
+
+    def __init__(self, words: int, group=None, device=None):
+        import torch
+        import torch.distributed as dist
+        self.words, self.group = int(words), group
+        self.world = dist.get_world_size(group) if group is not None else 1
+        self.rank = dist.get_rank(group) if group is not None else 0
+        if self.world > TBS_MAX_PEERS:
+            raise TbsError(f"fused combine supports at most {TBS_MAX_PEERS} ranks")
+        dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+        with torch.cuda.device(dev):
+            p, h = ctypes.c_void_p(), ctypes.create_string_buffer(64)
+            _check(lib().tbs_peer_alloc(self.words * 8, ctypes.byref(p), h), "tbs_peer_alloc")
+            self._own = p.value
+            handles = [None] * self.world
+            if group is not None:
+                dist.all_gather_object(handles, h.raw, group=group)
+            else:
+                handles[0] = h.raw
+            self._opened, ptrs = [], []
+            for r, hr in enumerate(handles):
+                if r == self.rank:
+                    ptrs.append(self._own)
+                else:
+                    q = ctypes.c_void_p()
+                    _check(lib().tbs_peer_open(hr, ctypes.byref(q)), "tbs_peer_open")
+                    self._opened.append(q.value)
+                    ptrs.append(q.value)
+        self.ptrs = (ctypes.c_void_p * self.world)(*ptrs)
+        self.local = torch.as_tensor(_CudaArray(self._own, self.words), device=dev)
+
+    def _barrier(self):
+        if self.group is not None:
+            import torch.distributed as dist
+            dist.barrier(group=self.group)
+
+    def begin(self, stream=None):
+        import torch
+        st = stream if stream is not None else torch.cuda.current_stream(self.local.device)
+        with torch.cuda.stream(st):
+            self.local.zero_()
+        st.synchronize()
+        self._barrier()
+
+    def finish(self, stream=None, out=None):
+        import torch
+        st = stream if stream is not None else torch.cuda.current_stream(self.local.device)
+        st.synchronize()
+        self._barrier()
+        with torch.cuda.stream(st):
+            return self.local.clone() if out is None else out.copy_(self.local)
+
+    def close(self):
+        if self._own is None:
+            return
+        for q in self._opened:
+            lib().tbs_peer_close(q)
+        self._barrier()   # no rank frees its buffer while a peer may still map it
+        lib().tbs_peer_free(self._own)
+        self._own, self._opened = None, []
+
+
+class _CudaArray:
+    """__cuda_array_interface__ view of a raw int64 device buffer (no copy)."""
+
+    def __init__(self, ptr, words):
+        self.__cuda_array_interface__ = {"shape": (words,), "typestr": "<i8", "data": (ptr, False), "version": 3}
+
+
+def _fused(a, sink):
+    if sink is not None:
+        a.flags |= TBS_OUT_PEERS
+        a.out_peers, a.n_out_peers = sink.ptrs, sink.world
+    return a
+
+
 def combine(partial, group=None):
     """The method's one exchange step: sum the per-rank int64 partial
     histograms / counts with a single all_reduce (NCCL over NVLink on GPUs). Integer
@@ -165,26 +261,36 @@ def _args(points, rows, flags, stream, events):
 
 
 def sdh(points, bucket_width: float, nbuckets: int, *, rows=None, lattice: bool = False, hist_mode=None,
-        force_clamp: bool = False, out=None, stream=None, events=None, group=None):
+        force_clamp: bool = False, out=None, stream=None, events=None, group=None, sink=None):
     """Spatial distance histogram (Type-II). Returns int64[nbuckets] on points.device.
 
     rows=(b, e): only anchors i in [b, e) (with all partners j > i). lattice=True:
     exact integer bucketing (integer-valued points, bucket_width = m * 2^-j).
     group: a torch.distributed process group: each rank computes its pair-balanced
-    strip (rank_rows) and the partial histograms are summed with one all_reduce.
+    strip (rank_rows) and the partial histograms are summed with one all_reduce, or, with
+    sink=PeerSink(nbuckets, group), by the kernels' own flush into every rank's buffer.
     """
     torch = _torch()
     flags = (TBS_EXACT_LATTICE if lattice else 0) | HIST_MODES[hist_mode] | (TBS_FORCE_CLAMP if force_clamp else 0)
     a, _ = _args(points, partition(points.shape[0], group, rows), flags, stream, events)
+    if sink is not None:            # fused combine: the kernels' flush is the all-reduce
+        sink.begin(stream)
+        _check(lib().tbs_sdh_ex(ctypes.byref(_fused(a, sink)), float(bucket_width), int(nbuckets), None), "tbs_sdh_ex")
+        return sink.finish(stream, out)
     h = out if out is not None else torch.empty(nbuckets, dtype=torch.int64, device=points.device)
     _check(lib().tbs_sdh_ex(ctypes.byref(a), float(bucket_width), int(nbuckets), h.data_ptr()), "tbs_sdh_ex")
     return combine(h, group)
 
 
-def pcf(points, radius: float, *, rows=None, out=None, stream=None, events=None, group=None):
-    """2-point correlation count (Type-I): #{i<j : d < radius}, int64[1] on points.device."""
+def pcf(points, radius: float, *, rows=None, out=None, stream=None, events=None, group=None, sink=None):
+    """2-point correlation count (Type-I): #{i<j : d < radius}, int64[1] on points.device.
+    sink=PeerSink(1, group): fused combine (see sdh)."""
     torch = _torch()
     a, _ = _args(points, partition(points.shape[0], group, rows), 0, stream, events)
+    if sink is not None:
+        sink.begin(stream)
+        _check(lib().tbs_pcf_ex(ctypes.byref(_fused(a, sink)), float(radius), None), "tbs_pcf_ex")
+        return sink.finish(stream, out)
     c = out if out is not None else torch.empty(1, dtype=torch.int64, device=points.device)
     _check(lib().tbs_pcf_ex(ctypes.byref(a), float(radius), c.data_ptr()), "tbs_pcf_ex")
     return combine(c, group)

@@ -22,6 +22,7 @@
 #include "tbs_knn.cuh"
 
 using namespace tbs;
+static_assert(kMaxPeers == TBS_MAX_PEERS, "peer sink size");
 
 // Pair-engine configurations per output type: anchors/thread, partner chunk, CTAs/SM
 // (A/B-tunable with -D at build time, see tools/build_ab.py).
@@ -155,7 +156,8 @@ int D_of(const tbs_args* a) { return a->dim <= 3 ? 3 : 4; }
 // Persistent grid for a pair-kernel instantiation: SMs x resident CTAs (at most one CTA per item).
 template <class Op, int D, class C, int VSET = 0x1F>
 int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op& op, const uint32_t* bbox,
-                cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee, bool first_launch_on_scratch = true) {
+                cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee, bool first_launch_on_scratch = true,
+                const OutSink& sink = OutSink{}) {
   // bbox may be nulled (TBS_FORCE_CLAMP); the 64-byte block always follows the SoA copy
   const uint32_t* bbox_block = reinterpret_cast<const uint32_t*>(soa + (size_t)D_of(a) * pad_rows(a->n));
   auto kern = pair_kernel<Op, D, C, VSET>;
@@ -189,7 +191,7 @@ int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op
   static const bool trace_on = getenv("TBS_TRACE") != nullptr;  // debug: CTA residency trace to stderr
   if (trace_on) TBS_CUDA(cudaMalloc(&g.trace, (size_t)grid * 3 * 8));
   if (eb) TBS_CUDA(cudaEventRecord(eb, st));
-  kern<<<(unsigned)grid, kThreads, (size_t)smem, st>>>(soa, g, op, bbox);
+  kern<<<(unsigned)grid, kThreads, (size_t)smem, st>>>(soa, g, op, bbox, sink);
   TBS_CUDA(cudaGetLastError());
   g_launches.fetch_add(1);
   if (ee) TBS_CUDA(cudaEventRecord(ee, st));
@@ -219,8 +221,15 @@ int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op
   return TBS_OK;
 }
 
-int validate_common(const tbs_args* a) {
+int validate_common(const tbs_args* a, bool peers_ok = false) {
   if (!a) return fail(TBS_EINVAL, "args is NULL");
+  if (a->flags & TBS_OUT_PEERS) {
+    if (!peers_ok) return fail(TBS_EUNSUPPORTED, "TBS_OUT_PEERS: SDH and 2PCF only");
+    if (a->n_out_peers < 1 || a->n_out_peers > kMaxPeers || !a->out_peers)
+      return fail(TBS_EINVAL, "TBS_OUT_PEERS needs 1..%d out_peers", kMaxPeers);
+    for (int w = 0; w < a->n_out_peers; ++w)
+      if (!a->out_peers[w]) return fail(TBS_EINVAL, "out_peers[%d] is NULL", w);
+  }
   if (a->n < 0 || a->n > TBS_MAX_N) return fail(TBS_EINVAL, "n = %lld outside [0, 2^30]", (long long)a->n);
   if (a->dim < 1 || a->dim > 4) return fail(TBS_EINVAL, "dim = %d outside [1, 4]", a->dim);
   if (a->row_begin < 0 || a->row_end < a->row_begin || a->row_end > a->n)
@@ -248,6 +257,19 @@ int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long 
   return TBS_OK;
 }
 
+// Output sink of a Type-I/II call: the caller's buffer, or every rank's (TBS_OUT_PEERS).
+OutSink make_sink(const tbs_args* a, unsigned long long* own) {
+  OutSink o{};
+  if (a->flags & TBS_OUT_PEERS) {
+    o.n = a->n_out_peers;
+    for (int w = 0; w < o.n; ++w) o.p[w] = reinterpret_cast<unsigned long long*>(a->out_peers[w]);
+  } else {
+    o.n = 0;
+    o.p[0] = own;
+  }
+  return o;
+}
+
 // Decompose a dyadic width w = m * 2^-j (m odd or j = 0). Returns false if not dyadic.
 bool dyadic(float w, long long& m, int& j) {
   double x = (double)w;
@@ -273,19 +295,19 @@ struct SdhPlan {
 // not select exits at once (the work-queue counter is untouched by it).
 template <class Op, int D, class C, bool LAT>
 int launch_sdh(const Device& dev, const float* soa, const tbs_args* g, const Op& op, const uint32_t* bbox,
-               cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee) {
+               cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee, const OutSink& sink) {
   if constexpr (!LAT) {
-    return launch_pair<Op, D, C>(dev, soa, g, op, bbox, st, eb, ee);
+    return launch_pair<Op, D, C>(dev, soa, g, op, bbox, st, eb, ee, true, sink);
   } else {
-    int rc = launch_pair<Op, D, LatFastCfg, 0x11>(dev, soa, g, op, bbox, st, eb, nullptr);
+    int rc = launch_pair<Op, D, LatFastCfg, 0x11>(dev, soa, g, op, bbox, st, eb, nullptr, true, sink);
     if (rc) return rc;
-    return launch_pair<Op, D, C, 0xE>(dev, soa, g, op, bbox, st, nullptr, ee);
+    return launch_pair<Op, D, C, 0xE>(dev, soa, g, op, bbox, st, nullptr, ee, true, sink);
   }
 }
 
 template <int D, bool LAT>
 int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const uint32_t* bbox, const tbs_args* g, float w,
-                 long long m, int j, int nb, unsigned long long* hist, unsigned long long* part, int G, cudaStream_t st,
+                 long long m, int j, int nb, const OutSink& hist, unsigned long long* part, int G, cudaStream_t st,
                  cudaEvent_t eb, cudaEvent_t ee) {
   if (pl.global) {
     SdhGlobalOp<LAT> op{};
@@ -313,7 +335,6 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
     op.mj = (float)std::ldexp((double)m, -j);
     op.m = (int)m;
     op.sh = 2 * j;
-    op.hist = hist;
     // per item, a replica receives at most (32/R) lanes x kWarps x KA x TP increments
     if (LAT) ka_tp = std::max<long long>(ka_tp, (long long)LatFastCfg::KA * LatFastCfg::TP);
     const long long per_item = (long long)(32 / R) * kWarps * ka_tp;
@@ -331,7 +352,7 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
       const bool last = p + 1 == pl.passes;
       op.rows = last ? (nb - op.klo) + (LAT ? 0 : kGuard) : pl.pass_rows;
       rc = launch_pair<SdhSmemOp<0, LAT, true>, D, C>(dev, soa, g, op, bbox, st, p == 0 ? eb : nullptr,
-                                                       last ? ee : nullptr, p == 0);
+                                                       last ? ee : nullptr, p == 0, hist);
     }
     return rc;
   }
@@ -341,46 +362,47 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
       if constexpr (!LAT) {   // (lattice mode never takes the small-problem config)
         if (small) {
           fill(op, 32, (long long)SmallCfg::KA * SmallCfg::TP);
-          return launch_pair<SdhSmemOp<5, LAT>, D, SmallCfg>(dev, soa, g, op, bbox, st, eb, ee);
+          return launch_pair<SdhSmemOp<5, LAT>, D, SmallCfg>(dev, soa, g, op, bbox, st, eb, ee, true, hist);
         }
       }
       fill(op, 32, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<5, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<5, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
     }
     case 4: {
       SdhSmemOp<4, LAT> op{};
       fill(op, 16, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<4, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<4, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
     }
     case 3: {
       SdhSmemOp<3, LAT> op{};
       fill(op, 8, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<3, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<3, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
     }
     case 2: {
       SdhSmemOp<2, LAT> op{};
       fill(op, 4, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<2, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<2, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
     }
     case 1: {
       SdhSmemOp<1, LAT> op{};
       fill(op, 2, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<1, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<1, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
     }
     default: {
       SdhSmemOp<0, LAT> op{};
       fill(op, 1, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<0, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee);
+      return launch_sdh<SdhSmemOp<0, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
     }
   }
 }
 
 int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
-  int rc = validate_common(a);
+  int rc = validate_common(a, true);
   if (rc) return rc;
   if (nb < 1 || nb > TBS_MAX_BUCKETS) return fail(TBS_EINVAL, "nbuckets = %d outside [1, 2^24]", nb);
   if (!(w > 0.f) || !std::isfinite(w)) return fail(TBS_EINVAL, "bucket_width must be finite and > 0");
-  if (!hist) return fail(TBS_EINVAL, "hist is NULL");
+  const bool peers = (a->flags & TBS_OUT_PEERS) != 0;
+  if (!hist && !peers) return fail(TBS_EINVAL, "hist is NULL");
   const bool lattice = (a->flags & TBS_EXACT_LATTICE) != 0;
   long long m = 1;
   int j = 0;
@@ -393,9 +415,10 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   cudaStream_t st = (cudaStream_t)a->stream;
   auto* h = reinterpret_cast<unsigned long long*>(hist);
   if (a->n < 2 || a->row_begin >= a->row_end) {
-    TBS_CUDA(cudaMemsetAsync(h, 0, (size_t)nb * 8, st));
+    if (!peers) TBS_CUDA(cudaMemsetAsync(h, 0, (size_t)nb * 8, st));   // (fused combine: adds nothing)
     return TBS_OK;
   }
+  const OutSink sink = make_sink(a, h);
   // Output-stage plan: lane-private copies (R = 32) while they fit a 96 KB budget (two CTAs
   // per SM), then 4 replicas, then one copy per CTA; beyond that, global partial copies.
   SdhPlan pl{lattice, false, 5};
@@ -453,16 +476,17 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   }
   float* soa = nullptr;
   // Smem modes accumulate into hist: the loader zeroes it. Global mode zeroes the partials
-  // (the reduce kernel overwrites hist).
+  // (the reduce kernel overwrites hist). Fused combine: the callers zeroed every rank's buffer.
   uint32_t* bbox = nullptr;
-  rc = load_points(a, D, n_pad, &soa, pl.global ? part : h, pl.global ? zero_words : nb, st, &bbox);
+  rc = load_points(a, D, n_pad, &soa, pl.global ? part : (peers ? nullptr : h), pl.global ? zero_words : (peers ? 0 : nb),
+                   st, &bbox);
   if (a->flags & TBS_FORCE_CLAMP) bbox = nullptr;
   if (!rc) {
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
-    if (D == 3) rc = lattice ? sdh_dispatch<3, true>(dev, pl, soa, bbox, a, w, m, j, nb, h, part, G, st, eb, ee)
-                             : sdh_dispatch<3, false>(dev, pl, soa, bbox, a, w, m, j, nb, h, part, G, st, eb, ee);
-    else rc = lattice ? sdh_dispatch<4, true>(dev, pl, soa, bbox, a, w, m, j, nb, h, part, G, st, eb, ee)
-                      : sdh_dispatch<4, false>(dev, pl, soa, bbox, a, w, m, j, nb, h, part, G, st, eb, ee);
+    if (D == 3) rc = lattice ? sdh_dispatch<3, true>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee)
+                             : sdh_dispatch<3, false>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee);
+    else rc = lattice ? sdh_dispatch<4, true>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee)
+                      : sdh_dispatch<4, false>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee);
   }
   if (soa) cudaFreeAsync(soa, st);
   if (part) cudaFreeAsync(part, st);
@@ -470,35 +494,36 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
 }
 
 int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
-  int rc = validate_common(a);
+  int rc = validate_common(a, true);
   if (rc) return rc;
   if (!(r >= 0.f) || std::isinf(r)) return fail(TBS_EINVAL, "radius must be finite and >= 0");
-  if (!count) return fail(TBS_EINVAL, "count is NULL");
+  const bool peers = (a->flags & TBS_OUT_PEERS) != 0;
+  if (!count && !peers) return fail(TBS_EINVAL, "count is NULL");
   Device dev;
   if ((rc = current_device(dev))) return rc;
   cudaStream_t st = (cudaStream_t)a->stream;
   auto* c = reinterpret_cast<unsigned long long*>(count);
   if (a->n < 2 || a->row_begin >= a->row_end) {
-    TBS_CUDA(cudaMemsetAsync(c, 0, 8, st));
+    if (!peers) TBS_CUDA(cudaMemsetAsync(c, 0, 8, st));
     return TBS_OK;
   }
   const int D = a->dim <= 3 ? 3 : 4;
   float* soa = nullptr;
   uint32_t* bbox = nullptr;
-  rc = load_points(a, D, pad_rows(a->n), &soa, c, 1, st, &bbox);
+  rc = load_points(a, D, pad_rows(a->n), &soa, peers ? nullptr : c, peers ? 0 : 1, st, &bbox);
   if (!rc) {
     PcfOp op{};
     op.r2 = (float)((double)r * (double)r);
-    op.count = c;
+    const OutSink sink = make_sink(a, c);
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
     const bool small =
         make_geom(a->n, a->row_begin, a->row_end, PcfCfg::TA, PcfCfg::TP).items < (long long)small_items_per_sm() * dev.sms;
     if (small)
-      rc = D == 3 ? launch_pair<PcfOp, 3, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee)
-                  : launch_pair<PcfOp, 4, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee);
+      rc = D == 3 ? launch_pair<PcfOp, 3, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink)
+                  : launch_pair<PcfOp, 4, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink);
     else
-      rc = D == 3 ? launch_pair<PcfOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee)
-                  : launch_pair<PcfOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee);
+      rc = D == 3 ? launch_pair<PcfOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink)
+                  : launch_pair<PcfOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink);
   }
   if (soa) cudaFreeAsync(soa, st);
   return rc;
@@ -1001,6 +1026,39 @@ int tbs_rank_rows(int64_t n, int world, int rank, int64_t* row_begin, int64_t* r
   };
   *row_begin = boundary(rank);
   *row_end = boundary(rank + 1);
+  return TBS_OK;
+}
+
+int tbs_peer_alloc(uint64_t bytes, void** dev_ptr, void* handle) {
+  if (!dev_ptr || !handle || bytes == 0) return fail(TBS_EINVAL, "tbs_peer_alloc: bad arguments");
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, (size_t)bytes);
+  if (e == cudaErrorMemoryAllocation) return fail(TBS_ENOMEM, "tbs_peer_alloc: %s", cudaGetErrorString(e));
+  TBS_CUDA(e);
+  TBS_CUDA(cudaMemset(p, 0, (size_t)bytes));
+  cudaIpcMemHandle_t h;
+  TBS_CUDA(cudaIpcGetMemHandle(&h, p));
+  static_assert(sizeof(h) == 64, "IPC handle size");
+  memcpy(handle, &h, sizeof(h));
+  *dev_ptr = p;
+  return TBS_OK;
+}
+
+int tbs_peer_open(const void* handle, void** dev_ptr) {
+  if (!dev_ptr || !handle) return fail(TBS_EINVAL, "tbs_peer_open: bad arguments");
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle, sizeof(h));
+  TBS_CUDA(cudaIpcOpenMemHandle(dev_ptr, h, cudaIpcMemLazyEnablePeerAccess));
+  return TBS_OK;
+}
+
+int tbs_peer_close(void* dev_ptr) {
+  TBS_CUDA(cudaIpcCloseMemHandle(dev_ptr));
+  return TBS_OK;
+}
+
+int tbs_peer_free(void* dev_ptr) {
+  TBS_CUDA(cudaFree(dev_ptr));
   return TBS_OK;
 }
 

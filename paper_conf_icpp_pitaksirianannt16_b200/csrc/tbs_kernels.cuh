@@ -139,6 +139,30 @@ __device__ __forceinline__ float bbox_diameter(const uint32_t* __restrict__ bbox
 }
 
 // ------------------------------------------------------------------------------------
+// Where the Type-I / Type-II flushes land (a9, a12). n == 0: the caller's buffer p[0]
+// (device-scope atomics). n >= 1 (TBS_OUT_PEERS, the fused multi-GPU combine): every
+// rank's buffer p[0..n) — local or mapped from a peer GPU over NVLink by CUDA IPC — gets
+// every flushed partial with a system-scope atomic add, so when all ranks' kernels have
+// completed each buffer holds the all-reduced sum without a separate collective.
+// ------------------------------------------------------------------------------------
+constexpr int kMaxPeers = 16;
+struct OutSink {
+  unsigned long long* p[kMaxPeers];
+  int n;
+  __device__ __forceinline__ void add(long long k, unsigned long long v) const {
+    if (n == 0) {
+      atomicAdd(p[0] + k, v);
+    } else {
+      for (int w = 0; w < n; ++w) red_sys_add_u64(p[w] + k, v);
+    }
+  }
+  // After a CTA's last flush: order its remote adds before kernel completion is observed.
+  __device__ __forceinline__ void fence() const {
+    if (n != 0) __threadfence_system();
+  }
+};
+
+// ------------------------------------------------------------------------------------
 // Output-stage policies. Each provides:
 //   smem_bytes()                    dynamic shared memory it needs (host and device)
 //   init(smem), finish(smem)        zero / flush its private copies
@@ -178,7 +202,7 @@ struct SdhSmemOp {
   float scale_up;     // fp32(2^j / m) * (1 + 2^-17), rounded up (lattice fast variant)
   float scale_b;      // fp32(2^j / m) * (1 + 2^-19), rounded up (lattice bias-only variant)
   int m, sh;          // w = m * 2^-j, sh = 2 j            (lattice mode)
-  unsigned long long* hist;  // global u64 output [nb]
+  const OutSink* out; // global u64 output [nb] (or every rank's): the kernel's sink parameter
   float ymax;         // float: 2^23 + nb - 1 (clamp variant)
   int flush_every;    // items between overflow flushes
 
@@ -357,7 +381,7 @@ struct SdhSmemOp {
       for (int off = 1; off < R; off <<= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
       if ((lane & (R - 1)) == 0 && v != 0ull && e < total) {
         const int k = (e >> LOG2R) + (RANGED ? klo : 0);
-        atomicAdd(hist + (k < nb ? k : nb - 1), v);
+        out->add(k < nb ? k : nb - 1, v);
       }
     }
   }
@@ -369,7 +393,10 @@ struct SdhSmemOp {
       since = 0;
     }
   }
-  __device__ __forceinline__ void finish(unsigned char* smem) { flush(smem); }
+  __device__ __forceinline__ void finish(unsigned char* smem) {
+    flush(smem);
+    out->fence();
+  }
 };
 
 // Type-II, partially privatised GLOBAL histogram (large nb, or forced): G u64 copies in
@@ -383,6 +410,7 @@ struct SdhGlobalOp {
   unsigned long long* part;  // [G][nb]
   unsigned long long* mine;
   int flush_every;           // unused
+  const OutSink* out;        // unused (the reduce kernel writes the sink)
 
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) { mine = part + (size_t)(blockIdx.x % G) * nb; }
@@ -425,7 +453,7 @@ struct SdhGlobalOp {
 // count adds the sign bit of t: [s < r^2] with no compare instruction.
 struct PcfOp {
   float r2;
-  unsigned long long* count;
+  const OutSink* out;        // u64 count (or every rank's): the kernel's sink parameter
   uint32_t c;                // per-item counter (<= KA * TP)
   unsigned long long total;  // per-thread running total
 
@@ -460,7 +488,8 @@ struct PcfOp {
     if (threadIdx.x == 0) {
       unsigned long long s = 0;
       for (int w = 0; w < kWarps; ++w) s += red[w];
-      if (s) atomicAdd(count, s);
+      if (s) out->add(0, s);
+      out->fence();
     }
   }
 };
@@ -474,6 +503,7 @@ struct KdeOp {
   double* sum;              // global output (zeroed by the loader)
   float2 part;              // current group partial (two lanes of the packed pair)
   float tot, comp;          // Kahan running sum
+  const OutSink* out;       // unused
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) {
     part = make_float2(0.f, 0.f);
@@ -579,7 +609,8 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
 // footprint can be compiled (and made resident) on its own and launched beside the rest.
 template <class Op, int D, class C, int VSET = 0x1F>
 __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __restrict__ soa, Geom g, Op op,
-                                                            const uint32_t* __restrict__ bbox) {
+                                                            const uint32_t* __restrict__ bbox,
+                                                            const __grid_constant__ OutSink sink) {
   unsigned char* smem = tbs_smem;
   const long long hbytes = (op.smem_bytes() + 127) & ~127ll;
   float* bufs = reinterpret_cast<float*>(smem + hbytes);
@@ -589,6 +620,7 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
 
   unsigned long long t_start = 0;
   if (g.trace != nullptr && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
+  op.out = &sink;   // (param space: the Op stays small, its copy lives in registers)
   op.init(smem);
   const int variant = op.variant(bbox, D);
   if (!((VSET >> variant) & 1)) return;   // CTA-uniform: another launch owns this variant
@@ -719,12 +751,14 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
 // Sum G partial global copies into the output (one thread per bin, the paper's
 // reduction kernel K13, L778-782).
 __global__ void reduce_partials(const unsigned long long* __restrict__ part, int G, int nb,
-                                unsigned long long* __restrict__ hist) {
+                                OutSink out) {
   for (int k = blockIdx.x * blockDim.x + threadIdx.x; k < nb; k += gridDim.x * blockDim.x) {
     unsigned long long s = 0;
     for (int gi = 0; gi < G; ++gi) s += part[(size_t)gi * nb + k];
-    hist[k] = s;
+    if (out.n == 0) out.p[0][k] = s;      // overwrite: no zeroing of the output needed
+    else if (s) out.add(k, s);
   }
+  out.fence();
 }
 
 // ------------------------------------------------------------------------------------

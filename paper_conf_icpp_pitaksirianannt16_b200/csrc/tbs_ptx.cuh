@@ -64,6 +64,10 @@ __device__ __forceinline__ void red_smem_inc_if(uint32_t addr, bool c) {
       "r"((int)c));
 }
 // Global u64 increment (partially privatised global histogram, SASS: REDG.E.ADD.64).
+// System-scope u64 add (peer memory mapped over NVLink / CUDA IPC: the fused combine).
+__device__ __forceinline__ void red_sys_add_u64(unsigned long long* addr, unsigned long long v) {
+  asm volatile("red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(addr), "l"(v) : "memory");
+}
 __device__ __forceinline__ void red_gmem_inc64(unsigned long long* addr) {
   asm volatile("red.global.add.u64 [%0], 1;" ::"l"(addr) : "memory");
 }

@@ -85,6 +85,27 @@ def test_pcf_and_matrix_einval(L):
     assert L.tbs_pairmatrix_ex(ctypes.byref(a), tbs._Kernel(0, 1.0), None) == tbs.TBS_EINVAL
 
 
+def test_out_peers_validation(L):
+    """TBS_OUT_PEERS (fused multi-GPU combine): 1..16 non-NULL peer buffers, SDH and 2PCF only;
+    checked before any device work (no GPU needed)."""
+    arr = (ctypes.c_void_p * 3)(1, 2, 3)
+    a = _args()
+    a.flags = tbs.TBS_OUT_PEERS
+    assert L.tbs_sdh_ex(ctypes.byref(a), 0.5, 8, None) == tbs.TBS_EINVAL       # n_out_peers = 0
+    a.out_peers, a.n_out_peers = arr, tbs.TBS_MAX_PEERS + 1
+    assert L.tbs_pcf_ex(ctypes.byref(a), 0.5, None) == tbs.TBS_EINVAL
+    arr[1] = None
+    a.n_out_peers = 3
+    assert L.tbs_sdh_ex(ctypes.byref(a), 0.5, 8, None) == tbs.TBS_EINVAL       # a NULL peer
+    assert "out_peers[1]" in tbs.last_error()
+    arr[1] = 2
+    c = np.zeros(1, np.float64)
+    assert L.tbs_kde_ex(ctypes.byref(a), 1.0, c.ctypes.data) == tbs.TBS_EUNSUPPORTED
+    assert L.tbs_pairmatrix_ex(ctypes.byref(a), tbs._Kernel(0, 1.0), c.ctypes.data) == tbs.TBS_EUNSUPPORTED
+    assert L.tbs_peer_alloc(0, ctypes.byref(ctypes.c_void_p()), ctypes.create_string_buffer(64)) == tbs.TBS_EINVAL
+    assert L.tbs_peer_open(None, ctypes.byref(ctypes.c_void_p())) == tbs.TBS_EINVAL
+
+
 @pytest.mark.parametrize("n", [0, 1, 2, 3, 7, 100, 2048, 4096, 1 << 20, 4194304, 1 << 30])
 @pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
 def test_rank_rows_partition(L, n, world):
