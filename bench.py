@@ -335,7 +335,8 @@ def main():
         bytes_ = rank_units * 4.0
         achieved = bytes_ / (kavg * 1e-3)
         roof = {"bound": "hbm", "achieved": achieved / 1e9, "peak": pk["hbm"] / 1e9, "unit": "GB/s",
-                "frac": achieved / pk["hbm"], "peak_source": pk["hbm_src"],
+                "frac": achieved / pk["hbm"], "peak_source": pk["hbm_src"] + " (a read+write copy; this kernel only writes)",
+                "frac_of_nominal": achieved / 7.7e12,   # HGX HBM3e 7.7 TB/s (B200_PROFILING.md), context
                 "algorithmic_bytes_per_launch": bytes_}
         if op == "pairmatrix_hd":
             # the Gram contraction: 2 d flops per entry on the bf16 tensor cores; the bound is
