@@ -19,7 +19,6 @@
 #include "tbs_kernels.cuh"
 #include "tbs_hd.cuh"
 #include "tbs_hd2.cuh"
-#include "tbs_hd3.cuh"
 #include "tbs_knn.cuh"
 
 using namespace tbs;
@@ -695,25 +694,7 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
                             : 2 * (int)std::min<long long>(ntiles, dev.sms / 2);   // CTA pairs
     const float cexp = (float)(-(double)k.gamma * 1.4426950408889634);
     const int kblocks = dp / hd::kKBlock;
-    // A-stationary CTA pairs (tbs_hd3.cuh, opt-in with TBS_HD_AST=1, 128 < d <= 512): each
-    // pair keeps its A half resident per work unit and streams only B, halving the L2 operand
-    // traffic per tile — measured SLOWER at 64K x 512 (4.64 vs 4.12 ms): the hd2 kernel is
-    // not bound by L2 operand traffic, so hd2 stays the default.
-    static const int ast_env = [] { const char* e = getenv("TBS_HD_AST"); return e ? atoi(e) : 0; }();
-    const bool ast = !one_sm && ast_env != 0 && kblocks > 2 && kblocks <= hd3::kMaxKBlocks;
-    const int smem = (one_sm ? hd::Smem::BYTES : ast ? hd3::Smem::BYTES : hd2::Smem::BYTES) + 1024;
-    // A-stationary units: (tile row, one of `segs` column segments), chosen to balance units
-    // over clusters while keeping units long (an A refill per unit: 1/tiles-per-unit extra).
-    int segs = 1;
-    if (ast) {
-      const int C = grid / 2;
-      double best = -1.0;
-      for (int sg = 1; sg <= std::min(tiles_j, 64); ++sg) {
-        const long long U = (long long)tiles_i * sg;
-        const double eff = (double)U / (double)(((U + C - 1) / C) * C) / (1.0 + (double)sg / tiles_j);
-        if (eff > best + 1e-9) { best = eff; segs = sg; }
-      }
-    }
+    const int smem = (one_sm ? hd::Smem::BYTES : hd2::Smem::BYTES) + 1024;
     // CTA-pair tile raster: bands of `band` tile rows walked column by column, tiles dealt
     // round-robin over clusters (0: contiguous row-major range per cluster). TBS_HD_BAND overrides.
     static const int band_env = [] { const char* e = getenv("TBS_HD_BAND"); return e ? atoi(e) : -1; }();
@@ -726,10 +707,7 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
     auto launch = [&](auto kern) -> int {
       TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
       if (eb) TBS_CUDA(cudaEventRecord(eb, st));
-      if constexpr (std::is_same<decltype(kern), decltype(&hd3::hd_ast_kernel<0>)>::value)
-        kern<<<grid, hd3::kThreads, smem, st>>>(tmap, tmap_out, use_tma_store, norms, (int)n, kblocks, I0, tiles_i,
-                                                tiles_j, segs, (int)rb, (int)re, cexp, out);
-      else if constexpr (std::is_same<decltype(kern), decltype(&hd2::hd_pair_kernel<0>)>::value)
+      if constexpr (std::is_same<decltype(kern), decltype(&hd2::hd_pair_kernel<0>)>::value)
         kern<<<grid, hd2::kThreads, smem, st>>>(tmap, tmap_out, use_tma_store, norms, (int)n, kblocks, I0, tiles_i,
                                                 tiles_j, (int)rb, (int)re, cexp, out, band);
       else
@@ -744,10 +722,6 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
       rc = k.type == 0 ? launch(hd::hd_pairmatrix_kernel<0>)
            : k.type == 1 ? launch(hd::hd_pairmatrix_kernel<1>)
                          : launch(hd::hd_pairmatrix_kernel<2>);
-    else if (ast)
-      rc = k.type == 0 ? launch(hd3::hd_ast_kernel<0>)
-           : k.type == 1 ? launch(hd3::hd_ast_kernel<1>)
-                         : launch(hd3::hd_ast_kernel<2>);
     else
       rc = k.type == 0 ? launch(hd2::hd_pair_kernel<0>)
            : k.type == 1 ? launch(hd2::hd_pair_kernel<1>)

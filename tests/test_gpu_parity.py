@@ -434,34 +434,6 @@ def test_pairmatrix_hd_pair_tile_rows(tbs, rows, n):
     assert np.array_equal(part, full[rows[0]:rows[1]])
 
 
-def test_pairmatrix_hd_ast_equals_default(tbs, tmp_path):
-    """The opt-in A-stationary kernel (TBS_HD_AST=1, tbs_hd3.cuh) computes the same MMAs in
-    the same order and the same epilogue as the default CTA-pair kernel: bit-identical output
-    (several work units per cluster, a row range cutting pair tiles, n % 4 != 0)."""
-    import subprocess
-    import sys
-    import torch
-    code = (
-        "import sys, numpy as np, torch; sys.path.insert(0, %r);"
-        "import paper_conf_icpp_pitaksirianannt16_b200 as tbs;"
-        "x = torch.from_numpy(np.load(%r)).cuda().view(torch.bfloat16);"
-        "np.save(%r, np.stack([tbs.pairmatrix_hd(x, 0.01, kernel=k, rows=(100, 2900)).cpu().numpy()"
-        " for k in ('gaussian', 'dist')]))")
-    root = str(__import__("pathlib").Path(__file__).resolve().parents[1])
-    for n, d in [(3000, 200), (2950, 512)]:
-        rng = np.random.default_rng(n + d)
-        xb = _bf16_bits(rng.standard_normal((n, d)).astype(np.float32))
-        np.save(tmp_path / "x.npy", xb.view(np.int16))
-        env = dict(__import__("os").environ, TBS_HD_AST="1")
-        subprocess.run([sys.executable, "-c", code % (root, str(tmp_path / "x.npy"), str(tmp_path / "ast.npy"))],
-                       env=env, check=True, timeout=300)
-        ast = np.load(tmp_path / "ast.npy")
-        xt = torch.from_numpy(xb.view(np.int16)).cuda().view(torch.bfloat16)
-        for i, k in enumerate(("gaussian", "dist")):
-            ref = tbs.pairmatrix_hd(xt, 0.01, kernel=k, rows=(100, 2900)).cpu().numpy()
-            assert np.array_equal(ast[i], ref), (n, d, k)
-
-
 @pytest.mark.parametrize("n,d", [(9000, 64), (6000, 520), (6000, 448), (3000, 200)])
 def test_pairmatrix_hd_many_tiles_sampled(tbs, n, d):
     """More pair tiles than clusters (persistent round-robin / banded raster at d > 128):
