@@ -1,0 +1,2 @@
+set -x
+bash tools/sanitize.sh

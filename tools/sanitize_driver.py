@@ -27,6 +27,13 @@ out.append(float(tbs.pairmatrix(p[:1001], 1.0).sum().item()))
 out.append(float(tbs.pairmatrix(p[:1000], 1.0, kernel="dist").sum().item()))
 out.append(tbs.sdh(lat, 0.75, 80, lattice=True).sum().item())     # fast lattice variant, m = 3
 out.append(tbs.sdh(lat, 0.75, 7, lattice=True).sum().item())      # clamped two-sided fp32 variant
+out.append(tbs.sdh(lat, 0.09375, 256, lattice=True).sum().item())  # one-sided fp32 variant (X = 669)
+sink, csink = tbs.PeerSink(64), tbs.PeerSink(1)                    # fused combine (world 1)
+out.append(tbs.sdh(p, w, 64, sink=sink).sum().item())
+out.append(tbs.sdh(lat, 0.5, 64, lattice=True, hist_mode="global", sink=sink).sum().item())
+out.append(tbs.pcf(p, 0.05, rows=(7, 2000), sink=csink).item())
+sink.close()
+csink.close()
 out.append(float(tbs.kde(p, 1.0).item()))
 out.append(float(tbs.knn(p, 8)[1].sum().item()))
 out.append(float(tbs.knn(p, 5, rows=(3, 1800))[1].sum().item()))
