@@ -398,9 +398,9 @@ def main():
 
     # e2e: host buffers through the public API, H2D of the points and D2H of the result each step
     e2e = None
-    if op in ("sdh", "pcf", "kde", "knn"):
+    if op in ("sdh", "sdh_lattice", "pcf", "kde", "knn"):
         ph = torch.from_numpy(p_host).pin_memory()
-        if world == 1:
+        if world == 1 and op != "sdh_lattice":     # the simple host-pointer entry points
             hh = np.zeros(nb if op == "sdh" else 1, np.uint64)
             kh = np.zeros(1, np.float64)
 
@@ -420,6 +420,8 @@ def main():
                 d = ph.to(dev, non_blocking=True)
                 if op == "sdh":
                     r = tbs.sdh(d, w, nb, group=pg, sink=sink)
+                elif op == "sdh_lattice":
+                    r = tbs.sdh(d, w, nb, lattice=True, group=pg, sink=sink)
                 elif op == "kde":
                     r = tbs.kde(d, params["gamma"], group=pg)
                 elif op == "knn":

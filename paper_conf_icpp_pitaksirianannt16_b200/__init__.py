@@ -161,24 +161,44 @@ class PeerSink:
         if self.world > TBS_MAX_PEERS:
             raise TbsError(f"fused combine supports at most {TBS_MAX_PEERS} ranks")
         dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+        self._own, self._opened, err = None, [], None
         with torch.cuda.device(dev):
+            # every rank reaches every collective below, whatever fails locally, and all ranks
+            # agree at the end: either every mapping works or every rank raises
             p, h = ctypes.c_void_p(), ctypes.create_string_buffer(64)
-            _check(lib().tbs_peer_alloc(self.words * 8, ctypes.byref(p), h), "tbs_peer_alloc")
-            self._own = p.value
-            handles = [None] * self.world
-            if group is not None:
-                dist.all_gather_object(handles, h.raw, group=group)
+            if lib().tbs_peer_alloc(self.words * 8, ctypes.byref(p), h) == TBS_OK:
+                self._own = p.value
             else:
-                handles[0] = h.raw
-            self._opened, ptrs = [], []
+                err = "tbs_peer_alloc: " + last_error()
+            handles = [None] * self.world
+            mine = h.raw if self._own is not None else None
+            if group is not None:
+                dist.all_gather_object(handles, mine, group=group)
+            else:
+                handles[0] = mine
+            ptrs = []
             for r, hr in enumerate(handles):
                 if r == self.rank:
                     ptrs.append(self._own)
+                elif hr is None or err is not None:
+                    err = err or f"rank {r} has no buffer"
+                    ptrs.append(None)
                 else:
                     q = ctypes.c_void_p()
-                    _check(lib().tbs_peer_open(hr, ctypes.byref(q)), "tbs_peer_open")
-                    self._opened.append(q.value)
-                    ptrs.append(q.value)
+                    if lib().tbs_peer_open(hr, ctypes.byref(q)) == TBS_OK:
+                        self._opened.append(q.value)
+                        ptrs.append(q.value)
+                    else:
+                        err = "tbs_peer_open: " + last_error()
+                        ptrs.append(None)
+            if group is not None:
+                ok = torch.tensor([0 if err else 1], dtype=torch.int32, device=dev if dist.get_backend(group) == "nccl" else "cpu")
+                dist.all_reduce(ok, op=dist.ReduceOp.MIN, group=group)
+                if not int(ok.item()) and err is None:
+                    err = "another rank could not map the peer buffers"
+            if err is not None:
+                self.close()
+                raise TbsError(f"fused combine unavailable: {err}")
         self.ptrs = (ctypes.c_void_p * self.world)(*ptrs)
         self.local = torch.as_tensor(_CudaArray(self._own, self.words), device=dev)
 
@@ -204,12 +224,15 @@ class PeerSink:
             return self.local.clone() if out is None else out.copy_(self.local)
 
     def close(self):
-        if self._own is None:
+        """Collective over the group (every rank calls it once)."""
+        if getattr(self, "_closed", False):
             return
+        self._closed = True
         for q in self._opened:
             lib().tbs_peer_close(q)
         self._barrier()   # no rank frees its buffer while a peer may still map it
-        lib().tbs_peer_free(self._own)
+        if self._own is not None:
+            lib().tbs_peer_free(self._own)
         self._own, self._opened = None, []
 
 
