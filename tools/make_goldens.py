@@ -25,6 +25,10 @@ GOLDENS = {
     "pcf_clustered_n1048576_r0.03_seed3": dict(op="pcf", kind="clustered", n=1 << 20, seed=3, r=0.03),
     # BASELINE.json configs[3] recipe at full size: SDH N=2M uniform, 16384 buckets (seed 4)
     "sdh_uniform_n2097152_nb16384_seed4": dict(op="sdh", kind="uniform", n=1 << 21, seed=4, nb=16384),
+    # the north-star line at full size: SDH N=4M uniform, 256 buckets (seed 6)
+    "sdh_uniform_n4194304_nb256_seed6": dict(op="sdh", kind="uniform", n=1 << 22, seed=6, nb=256),
+    # BASELINE.json configs[2] at full size: 2PCF N=4M clustered, r = 0.03 (C3, seed 3)
+    "pcf_clustered_n4194304_r0.03_seed3": dict(op="pcf", kind="clustered", n=1 << 22, seed=3, r=0.03),
     # BASELINE.json configs[0]: SDH N=4096 uniform, 64 buckets (seed 1)
     "sdh_uniform_n4096_nb64_seed1": dict(op="sdh", kind="uniform", n=4096, seed=1, nb=64),
 }
