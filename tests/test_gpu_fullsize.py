@@ -66,6 +66,16 @@ def test_pcf_1m_clustered_vs_golden(tbs):
     check_pcf_float(c, gold["count"], gold["amb"])
 
 
+def test_pcf_4m_clustered_vs_golden(tbs):
+    """BASELINE.json configs[2] at full size: N=4M clustered, r=0.03 against the full oracle
+    count (tools/make_goldens.py, 8.8e12 pairs on the CPU)."""
+    gold = json.load(open(os.path.join(GOLD, "pcf_clustered_n4194304_r0.03_seed3.json")))
+    p = g.clustered(1 << 22, 3)
+    c = int(host(tbs.pcf(dev(p), 0.03))[0])
+    check_pcf_float(c, gold["count"], gold["amb"])
+    assert c > 2 ** 32
+
+
 def test_pcf_4m_clustered_strips(tbs):
     n = 1 << 22
     p = g.clustered(n, 3)

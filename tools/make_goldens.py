@@ -34,25 +34,72 @@ GOLDENS = {
 }
 
 
-def make(name):
+def part_rows(n, parts, k):
+    """Anchor rows of part k of `parts` with equal pair counts (sum over rows i of n-1-i):
+    boundary R solves R (2n - R - 1) / 2 = k/parts * n (n - 1) / 2. Parts are disjoint and
+    cover [0, n); the oracle's outputs over them add up to the full result."""
+    def bound(j):
+        if j == 0:
+            return 0
+        if j == parts:
+            return n
+        a = 2 * n - 1
+        return int(round((a - math.sqrt(a * a - 4.0 * j / parts * n * (n - 1))) / 2))
+    return bound(k), bound(k + 1)
+
+
+def make(name, part=None, parts=None, outdir=None):
+    """The golden `name`, or (part, parts) its k-th pair-balanced anchor-row part (for
+    oracle runs longer than one job; merged by merge())."""
     spec = GOLDENS[name]
     p = g.make(spec["kind"], spec["n"], spec["seed"])
+    rows = None if part is None else part_rows(spec["n"], parts, part)
     t0 = time.time()
     out = dict(name=name, spec=spec, generator="tbs_inputs." + spec["kind"], script="tools/make_goldens.py",
                threads=oracle.num_threads())
+    if rows is not None:
+        out.update(rows=list(rows), part=part, parts=parts)
     if spec["op"] == "sdh":
         w = float(np.float32(math.sqrt(3) / spec["nb"]))
-        h, a = oracle.sdh(p, w, spec["nb"])
+        h, a = oracle.sdh(p, w, spec["nb"], rows=rows)
         out.update(w=w, hist=[int(x) for x in h], amb=[int(x) for x in a])
     else:
-        c, a = oracle.pcf(p, spec["r"])
+        c, a = oracle.pcf(p, spec["r"], rows=rows)
         out.update(r=float(np.float32(spec["r"])), count=c, amb=a)
     out["oracle_seconds"] = round(time.time() - t0, 2)
+    fn = name + ("" if rows is None else f".part{part}of{parts}") + ".json"
+    with open(os.path.join(outdir or os.path.join(ROOT, "tests", "golden"), fn), "w") as f:
+        json.dump(out, f, indent=0)
+    print(fn, out["oracle_seconds"], "s")
+
+
+def merge(name, files):
+    """Sum the parts' oracle outputs (integer counts: order-independent) into the golden."""
+    ds = [json.load(open(f)) for f in files]
+    parts = ds[0]["parts"]
+    assert sorted(d["part"] for d in ds) == list(range(parts)) and all(d["name"] == name for d in ds)
+    out = dict(name=name, spec=ds[0]["spec"], generator=ds[0]["generator"], script="tools/make_goldens.py",
+               threads=ds[0]["threads"], merged_parts=[d["rows"] for d in sorted(ds, key=lambda d: d["part"])],
+               oracle_seconds=round(sum(d["oracle_seconds"] for d in ds), 2))
+    if "hist" in ds[0]:
+        out.update(w=ds[0]["w"], hist=[int(sum(v)) for v in zip(*(d["hist"] for d in ds))],
+                   amb=[int(sum(v)) for v in zip(*(d["amb"] for d in ds))])
+    else:
+        out.update(r=ds[0]["r"], count=sum(d["count"] for d in ds), amb=sum(d["amb"] for d in ds))
     with open(os.path.join(ROOT, "tests", "golden", name + ".json"), "w") as f:
         json.dump(out, f, indent=0)
-    print(name, out["oracle_seconds"], "s")
+    print(name, "merged from", len(ds), "parts")
 
 
 if __name__ == "__main__":
-    for nm in sys.argv[1:]:
-        make(nm)
+    # python tools/make_goldens.py NAME...                    full goldens
+    # python tools/make_goldens.py --part K PARTS OUTDIR NAME  one pair-balanced row part
+    # python tools/make_goldens.py --merge NAME PART_FILE...   sum the parts
+    a = sys.argv[1:]
+    if a and a[0] == "--part":
+        make(a[4], int(a[1]), int(a[2]), a[3])
+    elif a and a[0] == "--merge":
+        merge(a[1], a[2:])
+    else:
+        for nm in a:
+            make(nm)
