@@ -147,10 +147,13 @@ class PeerSink:
     ``finish()`` each rank's buffer holds the all-reduced result — the collective is fused
     into the kernels' flush instead of a separate NCCL all_reduce.
 
-    Protocol per result: ``begin(stream)`` zeroes this rank's buffer and waits (stream sync +
-    barrier) until every rank has zeroed; the compute call adds; ``finish(stream)`` waits
-    (stream sync + barrier) until every rank's kernels have completed and returns a copy of
-    the local buffer."""
+    Every rank holds two buffers (parity p = result index & 1), so one host barrier per
+    result suffices: ``begin(stream)`` enqueues the zeroing of this rank's OTHER-parity buffer
+    (the next result's); the compute call adds into every rank's parity-p buffer; ``finish``
+    syncs the stream, passes the barrier — after which every rank's adds for this result
+    have landed and every rank's next-parity buffer is zero, and nobody adds into it before
+    this barrier — and returns a copy of the local parity-p buffer (enqueued before the
+    zeroing of that buffer two results later)."""
 
     def __init__(self, words: int, group=None, device=None):
         import torch
@@ -166,7 +169,7 @@ class PeerSink:
             # every rank reaches every collective below, whatever fails locally, and all ranks
             # agree at the end: either every mapping works or every rank raises
             p, h = ctypes.c_void_p(), ctypes.create_string_buffer(64)
-            if lib().tbs_peer_alloc(self.words * 8, ctypes.byref(p), h) == TBS_OK:
+            if lib().tbs_peer_alloc(2 * self.words * 8, ctypes.byref(p), h) == TBS_OK:   # two parities, zeroed
                 self._own = p.value
             else:
                 err = "tbs_peer_alloc: " + last_error()
@@ -199,8 +202,19 @@ class PeerSink:
             if err is not None:
                 self.close()
                 raise TbsError(f"fused combine unavailable: {err}")
-        self.ptrs = (ctypes.c_void_p * self.world)(*ptrs)
-        self.local = torch.as_tensor(_CudaArray(self._own, self.words), device=dev)
+        self._ptrs = [(ctypes.c_void_p * self.world)(*[q + par * self.words * 8 for q in ptrs]) for par in (0, 1)]
+        both = torch.as_tensor(_CudaArray(self._own, 2 * self.words), device=dev)
+        self._local = (both[:self.words], both[self.words:])
+        self.parity = 0
+
+    @property
+    def ptrs(self):
+        """Every rank's parity-p buffer (the out_peers of the current result)."""
+        return self._ptrs[self.parity]
+
+    @property
+    def local(self):
+        return self._local[self.parity]
 
     def _barrier(self):
         if self.group is not None:
@@ -211,17 +225,17 @@ class PeerSink:
         import torch
         st = stream if stream is not None else torch.cuda.current_stream(self.local.device)
         with torch.cuda.stream(st):
-            self.local.zero_()
-        st.synchronize()
-        self._barrier()
+            self._local[self.parity ^ 1].zero_()
 
     def finish(self, stream=None, out=None):
         import torch
         st = stream if stream is not None else torch.cuda.current_stream(self.local.device)
         st.synchronize()
         self._barrier()
+        loc = self.local
+        self.parity ^= 1
         with torch.cuda.stream(st):
-            return self.local.clone() if out is None else out.copy_(self.local)
+            return loc.clone() if out is None else out.copy_(loc)
 
     def close(self):
         """Collective over the group (every rank calls it once)."""

@@ -108,6 +108,9 @@ def _ipc_worker(rank, world, port, q):
             hl = tbs.sdh(pl, 0.5, 80, lattice=True, group=dist.group.WORLD, sink=sink).cpu().tolist()
             hf = tbs.sdh(pc, float(np.float32(math.sqrt(3) / 80)), 80, group=dist.group.WORLD, sink=sink).cpu().tolist()
             c = int(tbs.pcf(pc, 0.03, group=dist.group.WORLD, sink=csink).cpu()[0])
+            # a third result on the same sink reuses parity 0 (zeroed during the second)
+            hl3 = tbs.sdh(pl, 0.5, 80, lattice=True, group=dist.group.WORLD, sink=sink).cpu().tolist()
+            assert hl3 == hl
             # the unfused path (all_reduce over gloo of CUDA tensors is unsupported: sum on host)
             part = tbs.sdh(pc, float(np.float32(math.sqrt(3) / 80)), 80, rows=tbs.partition(20000, dist.group.WORLD))
             part = part.cpu()
