@@ -141,6 +141,21 @@ def test_sdh_4m_uniform_strips_and_mass(tbs):
         check_sdh_float(hs, ho, amb)
 
 
+def test_sdh_4m_uniform_vs_golden_part(tbs):
+    """North-star workload at full size on its first pair-balanced anchor-row part (rows
+    [0, 1228483): half of the 8.8e12 pairs), against the CPU oracle's histogram of exactly
+    those pairs (tools/make_goldens.py --part 0 2, 43 min on 16 host threads)."""
+    gold = json.load(open(os.path.join(GOLD, "parts", "sdh_uniform_n4194304_nb256_seed6.part0of2.json")))
+    n = gold["spec"]["n"]
+    rb, re = gold["rows"]
+    p = g.uniform(n, gold["spec"]["seed"])
+    h = host(tbs.sdh(dev(p), gold["w"], 256, rows=(rb, re))).astype(np.uint64)
+    d = check_sdh_float(h, gold["hist"], gold["amb"])
+    # pairs (i, j), rb <= i < re, i < j < n
+    assert int(h.sum()) == sum(gold["hist"]) == (re - rb) * (2 * n - rb - re - 1) // 2
+    print("4M golden part 0:", d)
+
+
 def test_sdh_4m_lattice_exact(tbs):
     """L=160 lattice (N=4,096,000), w=1, 256 buckets: d_max = 275.4 so buckets >= 256 clamp
     into 255 (the clamp path); exact vs closed form."""
