@@ -13,7 +13,9 @@ Functions and their pins (tests/test_oracle_pins.py):
   pairmatrix     torch.cdist float64 (library routine), symmetry, diagonal
   lattice_closed brute force of sdh_lattice on permuted lattices
   kde            brute force (scipy pdist), closed form for coincident / two-point sets
-  rdf            hand-computed shells, uniform-cube law (g -> 1 - O(r) boundary deficit)
+  sdh_bands      = sdh (same loop) + the 5e-7 diagnostic band counts; band nesting, brute force
+  rdf            unit-ball volumes vs scipy.special.gamma, hand-computed 2-point shells in dims
+                 1-4, the uniform-hypercube covariogram law (Monte Carlo) in dims 1-4
   pairmatrix_hd  torch.cdist float64 on the decoded bf16 features, symmetry, diagonal
   knn            lexsort brute force, lattice neighbour shells (6/12/8), index tie-break, k > n-1
 Parity status: no worked example in PAPER.md prints values, so every pin is a
@@ -55,6 +57,8 @@ def _load():
         lib = ctypes.CDLL(_LIB)
         lib.oracle_sdh.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, ctypes.c_int, _i64, _i64,
                                    _u64p, _u64p]
+        lib.oracle_sdh_bands.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, ctypes.c_int, _i64, _i64,
+                                         _u64p, _u64p, _u64p]
         lib.oracle_sdh_lattice.argtypes = [_f32p, _i64, ctypes.c_int, _i64, ctypes.c_int, ctypes.c_int,
                                            _i64, _i64, _u64p]
         lib.oracle_pcf.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, _i64, _i64, _u64p, _u64p]
@@ -62,7 +66,8 @@ def _load():
                                           _f64p]
         lib.oracle_lattice_closed.argtypes = [_i64, _i64, ctypes.c_int, ctypes.c_int, _u64p, _i64, _u64p]
         lib.oracle_kde.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_double, _i64, _i64, _f64p]
-        lib.oracle_rdf.argtypes = [_u64p, ctypes.c_int, ctypes.c_int, ctypes.c_double, _i64, ctypes.c_double, _f64p]
+        lib.oracle_rdf.argtypes = [_u64p, ctypes.c_int, ctypes.c_int, ctypes.c_double, ctypes.c_double,
+                                   ctypes.c_double, _f64p]
         lib.oracle_pairmatrix_hd.argtypes = [ctypes.POINTER(ctypes.c_uint16), _i64, ctypes.c_int, ctypes.c_int,
                                              ctypes.c_double, _i64, _i64, _f64p]
         lib.oracle_knn.argtypes = [_f32p, _i64, ctypes.c_int, ctypes.c_int, _i64, _i64,
@@ -168,15 +173,49 @@ def kde(points, gamma, rows=None):
     return float(out[0])
 
 
-def rdf(hist, bucket_width, n, volume, dim=3):
-    """RDF g[k] = hist[k] / (C(n,2) shell_k / volume)."""
+def sdh_bands(points, bucket_width, nbuckets, rows=None):
+    """Float-mode SDH with both ambiguity bands: (hist, amb (1e-6), amb_diag (5e-7)), each
+    amb array uint64[nb+1] indexed by edge e = 1..nb-1 (SURVEY §8(c) diagnostic band)."""
+    p, n, dim = _pts(points)
+    rb, re = _rows(rows, n)
+    hist = np.zeros(nbuckets, np.uint64)
+    amb = np.zeros(nbuckets + 1, np.uint64)
+    amb2 = np.zeros(nbuckets + 1, np.uint64)
+    w = float(np.float32(bucket_width))
+    rc = _load().oracle_sdh_bands(_ptr(p, _f32p), n, dim, w, int(nbuckets), rb, re, _ptr(hist, _u64p),
+                                  _ptr(amb, _u64p), _ptr(amb2, _u64p))
+    if rc:
+        raise ValueError(f"oracle_sdh_bands: status {rc}")
+    return hist, amb, amb2
+
+
+def pairs_of_rows(n, rows=None):
+    """Pairs an anchor-row range [b, e) counts: sum_{i=b}^{e-1} (n - 1 - i)."""
+    b, e = _rows(rows, n)
+    return (e - b) * (2 * n - b - e - 1) // 2
+
+
+def rdf(hist, bucket_width, volume, dim=3, *, pairs):
+    """RDF g[k] = hist[k] / (pairs shell_k / volume) for the len(hist) real shells (R6)."""
     h = np.ascontiguousarray(hist, dtype=np.uint64)
     g = np.zeros(len(h), np.float64)
-    rc = _load().oracle_rdf(_ptr(h, _u64p), len(h), int(dim), float(np.float32(bucket_width)), int(n), float(volume),
-                            _ptr(g, _f64p))
+    rc = _load().oracle_rdf(_ptr(h, _u64p), len(h), int(dim), float(np.float32(bucket_width)), float(pairs),
+                            float(volume), _ptr(g, _f64p))
     if rc:
         raise ValueError(f"oracle_rdf: status {rc}")
     return g
+
+
+def rdf_points(points, bucket_width, nbuckets, volume, rows=None, lattice=None):
+    """The RDF pipeline of reading R6 on the oracle: SDH with nbuckets + 1 buckets (bucket nb
+    takes every d >= nb w), its first nb counts normalised by the pairs the rows count.
+    lattice=(m, j): exact-lattice SDH instead of float mode. Returns (g, hist[nb+1], amb)."""
+    p, n, dim = _pts(points)
+    if lattice is None:
+        h, amb = sdh(p, bucket_width, nbuckets + 1, rows=rows)
+    else:
+        h, amb = sdh_lattice(p, lattice[0], lattice[1], nbuckets + 1, rows=rows), None
+    return rdf(h[:nbuckets], bucket_width, volume, dim, pairs=pairs_of_rows(n, rows)), h, amb
 
 
 def pairmatrix_hd(features_bf16_bits, gamma, rows=None, ktype=0):

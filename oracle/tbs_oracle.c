@@ -66,20 +66,25 @@ static int check_common(const float* P, int64_t n, int dim, int64_t rb, int64_t 
  * amb (optional, length nb+1): amb[e] = #{i<j : |d_ij - e w| <= 1e-6 e w},
  * e = 1..nb-1 — the pairs whose bucket an fp32 evaluation may legitimately
  * place on either side of edge e (acceptance rule).
+ * amb_diag (optional, length nb+1): the same count for the narrower 5e-7 band,
+ * the diagnostic SURVEY §8(c) asks to report beside the 1e-6 rule ("also report,
+ * as a diagnostic, the mismatch count against a 5e-7 band").
  * w is the caller's fp32 bucket width, passed already widened to double.
  */
-int oracle_sdh(const float* P, int64_t n, int dim, double w, int nb,
-               int64_t row_begin, int64_t row_end, uint64_t* hist, uint64_t* amb) {
+int oracle_sdh_bands(const float* P, int64_t n, int dim, double w, int nb,
+                     int64_t row_begin, int64_t row_end, uint64_t* hist, uint64_t* amb, uint64_t* amb_diag) {
   if (check_common(P, n, dim, row_begin, row_end) || nb < 1 || !(w > 0.0) || isinf(w) || !hist)
     return ORACLE_EINVAL;
   int T = omp_get_max_threads();
   uint64_t* ph = (uint64_t*)calloc((size_t)T * nb, sizeof(uint64_t));
   uint64_t* pa = (uint64_t*)calloc((size_t)T * (nb + 1), sizeof(uint64_t));
-  if (!ph || !pa) { free(ph); free(pa); return ORACLE_ENOMEM; }
+  uint64_t* pd = (uint64_t*)calloc((size_t)T * (nb + 1), sizeof(uint64_t));
+  if (!ph || !pa || !pd) { free(ph); free(pa); free(pd); return ORACLE_ENOMEM; }
 #pragma omp parallel
   {
     uint64_t* h = ph + (size_t)omp_get_thread_num() * nb;
     uint64_t* a = pa + (size_t)omp_get_thread_num() * (nb + 1);
+    uint64_t* a2 = pd + (size_t)omp_get_thread_num() * (nb + 1);
 #pragma omp for schedule(guided)
     for (int64_t i = row_begin; i < row_end; ++i) {
       for (int64_t j = i + 1; j < n; ++j) {
@@ -89,17 +94,25 @@ int oracle_sdh(const float* P, int64_t n, int dim, double w, int nb,
         h[b] += 1;
         double e = rint(q);
         if (e >= 1.0 && e <= (double)(nb - 1) && fabs(d - e * w) <= 1e-6 * e * w) a[(int)e] += 1;
+        if (e >= 1.0 && e <= (double)(nb - 1) && fabs(d - e * w) <= 5e-7 * e * w) a2[(int)e] += 1;
       }
     }
   }
   memset(hist, 0, sizeof(uint64_t) * nb);
   if (amb) memset(amb, 0, sizeof(uint64_t) * (nb + 1));
+  if (amb_diag) memset(amb_diag, 0, sizeof(uint64_t) * (nb + 1));
   for (int t = 0; t < T; ++t) {
     for (int b = 0; b < nb; ++b) hist[b] += ph[(size_t)t * nb + b];
     if (amb) for (int e = 0; e <= nb; ++e) amb[e] += pa[(size_t)t * (nb + 1) + e];
+    if (amb_diag) for (int e = 0; e <= nb; ++e) amb_diag[e] += pd[(size_t)t * (nb + 1) + e];
   }
-  free(ph); free(pa);
+  free(ph); free(pa); free(pd);
   return ORACLE_OK;
+}
+
+int oracle_sdh(const float* P, int64_t n, int dim, double w, int nb,
+               int64_t row_begin, int64_t row_end, uint64_t* hist, uint64_t* amb) {
+  return oracle_sdh_bands(P, n, dim, w, nb, row_begin, row_end, hist, amb, NULL);
 }
 
 /* Exact integer square root: largest r with r*r <= S, for 0 <= S < 2^62. */
@@ -252,16 +265,20 @@ int oracle_kde(const float* P, int64_t n, int dim, double gamma, int64_t row_beg
 
 /*
  * Radial distribution function (Type-II, NEXT-1; "RDF, which outputs a
- * normalized form of SDH"): g[k] = hist[k] / ideal[k] with ideal[k] the expected count of an
- * ideal gas of n points in volume V, ideal[k] = C(n,2) * shell_k / V and shell_k the
- * dim-ball shell volume between k w and (k+1) w (unit-ball volumes 2, pi, 4 pi / 3, pi^2 / 2
- * for dim 1..4). The last (clamped, open) bucket is normalised by its closed shell too.
+ * normalized form of SDH"): g[k] = hist[k] / ideal[k], k = 0..nb-1, with ideal[k] the
+ * expected count of an ideal gas over the same pairs in volume V,
+ *   ideal[k] = pairs * shell_k / V,   shell_k = vol of the dim-ball shell k w <= r < (k+1) w
+ *            = c_dim ((k+1) w)^dim - c_dim (k w)^dim,
+ * unit-ball volumes c_1..c_4 = 2, pi, 4 pi / 3, pi^2 / 2. Reading R6: hist holds
+ * the counts of the nb real shells only (an SDH with nb+1 buckets whose clamp bucket nb is
+ * dropped), and `pairs` is the number of pairs that histogram counted (C(n,2) for the whole
+ * set, sum_{i in [b,e)} (n-1-i) for an anchor-row range).
  */
-int oracle_rdf(const uint64_t* hist, int nb, int dim, double w, int64_t n, double volume, double* g) {
-  if (!hist || !g || nb < 1 || dim < 1 || dim > 4 || !(w > 0.0) || !(volume > 0.0) || n < 0) return ORACLE_EINVAL;
+int oracle_rdf(const uint64_t* hist, int nb, int dim, double w, double pairs, double volume, double* g) {
+  if (!hist || !g || nb < 1 || dim < 1 || dim > 4 || !(w > 0.0) || !(volume > 0.0) || !(pairs >= 0.0))
+    return ORACLE_EINVAL;
   static const double unit_ball[5] = {0.0, 2.0, 3.14159265358979323846, 4.18879020478639098462,
                                       4.93480220054467930942};
-  const double pairs = (double)n * (double)(n - 1) / 2.0;
   for (int k = 0; k < nb; ++k) {
     const double shell = unit_ball[dim] * (pow((k + 1) * w, dim) - pow(k * w, dim));
     const double ideal = pairs * shell / volume;

@@ -281,24 +281,92 @@ def test_kde_bruteforce_and_closed_forms():
     assert abs(a - oracle.kde(p, 2.0)) < 1e-12 * oracle.kde(p, 2.0)
 
 
-def test_rdf_shells_and_uniform_cube():
-    h = np.array([10, 20, 30], np.uint64)
-    g3 = oracle.rdf(h, 0.5, 100, 8.0, dim=3)
-    pairs = 100 * 99 / 2
-    for k in range(3):
-        shell = 4 * math.pi / 3 * (((k + 1) * 0.5) ** 3 - (k * 0.5) ** 3)
-        assert abs(g3[k] - h[k] / (pairs * shell / 8.0)) < 1e-12
-    g1 = oracle.rdf(h, 0.5, 100, 8.0, dim=1)
-    assert abs(g1[1] - 20 / (pairs * 2 * 0.5 / 8.0)) < 1e-12
-    # uniform points in the unit cube: g(r) = P(bin) / (shell volume) -> 1 - (3/2)(r/1)*... at small r
-    p = g.uniform(4096, 1)
-    nb, w = 64, float(np.float32(math.sqrt(3) / 64))
-    hist, _ = oracle.sdh(p, w, nb)
-    gr = oracle.rdf(hist, w, 4096, 1.0)
-    expect = [(cube_cdf.F((k + 1) * w) - cube_cdf.F(k * w)) / (4 * math.pi / 3 * (((k + 1) * w) ** 3 - (k * w) ** 3))
-              for k in range(8)]
-    assert np.all(np.abs(gr[2:8] - np.array(expect[2:8])) < 0.05)             # statistical, boundary deficit
-    assert 0.85 < gr[3] < 1.0
+@pytest.mark.parametrize("dim", [1, 2, 3, 4])
+def test_rdf_unit_ball_vs_gamma_function(dim):
+    """The oracle's dim-ball volume c_d, read back through its API (one pair in shell 0 of
+    width 1, pairs = 1, V = 1 gives g[0] = 1 / c_d), equals pi^(d/2) / Gamma(d/2 + 1)
+    (scipy.special.gamma: a library routine the oracle does not use)."""
+    from scipy.special import gamma as G
+    g0 = oracle.rdf(np.array([1], np.uint64), 1.0, 1.0, dim, pairs=1)[0]
+    assert abs(1.0 / g0 - math.pi ** (dim / 2) / G(dim / 2 + 1)) < 1e-14
+
+
+@pytest.mark.parametrize("dim", [1, 2, 3, 4])
+def test_rdf_two_point_shell(dim):
+    """Hand case per dimension: two points 1.25 apart, w = 0.5, nb = 4, V = 10. The pair lies
+    in shell 2 = [1.0, 1.5); one pair counted, so g[2] = V / (c_d (1.5^d - 1^d)) and every
+    other shell is 0. The clamp bucket of the nb+1-bucket SDH stays empty (d < nb w = 2)."""
+    from scipy.special import gamma as G
+    p = np.zeros((2, dim), np.float32)
+    p[1, 0] = 1.25
+    gr, h, _ = oracle.rdf_points(p, 0.5, 4, 10.0)
+    assert h.tolist() == [0, 0, 1, 0, 0]
+    c = math.pi ** (dim / 2) / G(dim / 2 + 1)
+    expect = [0.0, 0.0, 10.0 / (c * (1.5 ** dim - 1.0)), 0.0]
+    np.testing.assert_allclose(gr, expect, rtol=1e-14, atol=0)
+    # a pair beyond nb w lands in the dropped clamp bucket, never in g
+    q = np.zeros((2, dim), np.float32)
+    q[1, 0] = 7.0
+    gq, hq, _ = oracle.rdf_points(q, 0.5, 4, 10.0)
+    assert hq.tolist() == [0, 0, 0, 0, 1] and not gq.any()
+
+
+def test_rdf_row_range_pairs():
+    """An anchor-row strip is normalised by the pairs that strip counts: strips
+    of a partition give g_strip * pairs_strip that sum to g_full * pairs_full."""
+    p = g.uniform(900, 31)
+    w, nb = 0.05, 20
+    full, _, _ = oracle.rdf_points(p, w, nb, 1.0)
+    acc = np.zeros(nb)
+    for rows in ((0, 100), (100, 450), (450, 900)):
+        gs, _, _ = oracle.rdf_points(p, w, nb, 1.0, rows=rows)
+        acc += gs * oracle.pairs_of_rows(900, rows)
+    assert oracle.pairs_of_rows(900) == 900 * 899 // 2
+    np.testing.assert_allclose(acc, full * (900 * 899 // 2), rtol=1e-12)
+
+
+def covariogram_g(dim, r0, r1, m=400000, seed=0):
+    """Expected RDF of uniform points in the unit dim-cube over the shell [r0, r1): the mean of
+    the cube's set covariogram prod_c (1 - |u_c|)^+ over points u uniform in the shell
+    (E h_k / pairs = int_shell prod_c (1 - |u_c|)^+ du). Monte Carlo, independent of the oracle."""
+    rng = np.random.default_rng(seed)
+    r = (r0 ** dim + rng.random(m) * (r1 ** dim - r0 ** dim)) ** (1.0 / dim)
+    v = rng.standard_normal((m, dim))
+    u = v / np.linalg.norm(v, axis=1, keepdims=True) * r[:, None]
+    f = np.prod(np.clip(1.0 - np.abs(u), 0.0, None), axis=1)
+    return f.mean(), f.std() / math.sqrt(m)
+
+
+@pytest.mark.parametrize("dim", [1, 2, 3, 4])
+def test_rdf_uniform_hypercube_law(dim):
+    """Uniform points in the unit dim-cube (V = 1): the oracle's g over 8 seeds agrees with the
+    covariogram law (Monte Carlo above) within 5 standard errors (the seeds' spread) plus the
+    Monte Carlo error. A wrong ball constant, exponent or pair count shifts g by >= 10 %."""
+    n, nb = 2000, 8
+    w = {1: 0.02, 2: 0.02, 3: 0.04, 4: 0.06}[dim]
+    gs = np.array([oracle.rdf_points(g.uniform(n, 100 + s, dim), w, nb, 1.0)[0] for s in range(8)])
+    mean, se = gs.mean(0), gs.std(0, ddof=1) / math.sqrt(len(gs))
+    for k in range(1, nb):
+        ex, mc = covariogram_g(dim, k * w, (k + 1) * w, seed=k)
+        assert abs(mean[k] - ex) <= 5 * se[k] + 5 * mc + 1e-3, (dim, k, mean[k], ex, se[k])
+    assert 0.5 < mean[1:].mean() < 1.0      # boundary deficit: g < 1 for a finite cube
+
+
+def test_sdh_bands_bruteforce():
+    """oracle.sdh_bands: same histogram and 1e-6 band as oracle.sdh, and the 5e-7 diagnostic
+    band equals a scipy pdist brute-force count; the bands nest."""
+    p = g.uniform(1500, 41)
+    nb = 16384
+    w = float(np.float32(math.sqrt(3) / nb))
+    h, a, a2 = oracle.sdh_bands(p, w, nb)
+    h1, a1 = oracle.sdh(p, w, nb)
+    assert h.tolist() == h1.tolist() and a.tolist() == a1.tolist()
+    _, d = brute_sdh(p, w, nb)
+    wd = np.float64(np.float32(w))
+    e = np.rint(d / wd)
+    ok = (e >= 1) & (e <= nb - 1) & (np.abs(d - e * wd) <= 5e-7 * e * wd)
+    assert a2.tolist() == np.bincount(e[ok].astype(np.int64), minlength=nb + 1).tolist()
+    assert np.all(a2 <= a) and a2.sum() > 100 and a.sum() > a2.sum()
 
 
 # ---------------------------------------------------------------- NEXT-3: high-dimensional Type-III (bf16 features)
