@@ -6,10 +6,17 @@ full pass of the hot path: SoA loader -> triangular pair kernel with the privati
 shared-memory histogram -> u64 flush (-> NCCL all_reduce of the histogram for N>1).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NAME] [--impl tbs|reference]
+                    [--combine nccl|fused] [--dry-run]
 
-Multi-GPU: launched by torchrun, one rank per GPU; each rank computes its
-pair-balanced anchor strip (tbs_rank_rows) and the ranks sum their histograms with
-one all_reduce (strong scaling: the problem is fixed). Time = CUDA events on the
+Multi-GPU: one rank per GPU. Under torchrun (WORLD_SIZE set) the ranks are torchrun's and
+WORLD_SIZE must equal --gpus; a plain `python bench.py --gpus N` (N > 1) re-launches itself
+through torch.distributed.run with N local ranks. Each rank computes its pair-balanced anchor
+strip (tbs_rank_rows) and the ranks sum their histograms with one NCCL all_reduce
+(--combine nccl, the default and the north star's path) or with the kernels' own flush into
+every rank's buffer over peer memory (--combine fused, TBS_OUT_PEERS). Strong scaling: the
+problem is fixed. NCCL's INIT log goes to stderr (NCCL_DEBUG=INFO, NCCL_DEBUG_SUBSYS=INIT
+unless set) so the communicator's ranks can be counted. --dry-run: no GPU work — the ranks
+join a gloo group, check the world size and print their row strips (CPU test of the launch). Time = CUDA events on the
 launching stream around exactly K steps, barrier + synchronize on both sides, max
 over ranks. The L2 (126 MB) is flushed between steps by writing 256 MiB; the
 inputs (12 MiB) are smaller than L2 and the flush is inside the timed region.
@@ -24,7 +31,6 @@ import json
 import math
 import os
 import statistics
-import subprocess
 import sys
 import time
 
@@ -84,40 +90,75 @@ def units_of(op, n):
 
 # ------------------------------------------------------------------ clocks sampler
 class Clocks:
-    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+    """SM clock + clock-event reasons sampled DURING the timed region.
 
-    def __init__(self, gpu_index):
-        self.p = None
-        self.out = os.path.join("/tmp", f"tbs_clocks_{os.getpid()}.csv")
+    A background thread polls NVML every 5 ms (the GPU is found by PCI bus id, so
+    CUDA_VISIBLE_DEVICES remappings do not matter); `mark(True)` / `mark(False)` bracket the
+    timed region on the host. Runs shorter than a few NVML periods still get their samples:
+    the sampler is started (and has produced a sample) before the region opens, and the
+    samples inside the bracket, plus the last one before and the first one after it, are
+    reported, with `window_ms` and `samples` so a reader can judge them (None if NVML is
+    unavailable)."""
+    REASONS = {0x4: "sw_power_cap", 0x8: "hw_slowdown", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown"}
+
+    def __init__(self, torch_device):
+        import threading
+        self.rows, self.t0, self.t1, self.src = [], None, None, "nvml"
+        self._stop = threading.Event()
         try:
-            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                                       "-i", str(gpu_index), "-lms", "100"], stdout=open(self.out, "w"),
-                                      stderr=subprocess.DEVNULL)
-        except Exception:
-            self.p = None
+            import pynvml as nv
+            nv.nvmlInit()
+            h = None
+            try:
+                import torch
+                pr = torch.cuda.get_device_properties(torch_device)
+                bus = f"{pr.pci_domain_id:08x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+                h = nv.nvmlDeviceGetHandleByPciBusId_v2(bus)
+            except Exception:   # noqa: BLE001 — fall back to the visible index
+                h = nv.nvmlDeviceGetHandleByIndex(torch_device.index or 0)
+            self.max_mhz = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+
+            def poll():
+                while not self._stop.is_set():
+                    try:
+                        self.rows.append((time.perf_counter(), nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM),
+                                          nv.nvmlDeviceGetCurrentClocksEventReasons(h)))
+                    except Exception:   # noqa: BLE001
+                        pass
+                    self._stop.wait(0.005)
+            self.th = threading.Thread(target=poll, daemon=True)
+            self.th.start()
+            t_end = time.perf_counter() + 2.0
+            while not self.rows and time.perf_counter() < t_end:
+                time.sleep(0.002)
+        except Exception:   # noqa: BLE001
+            self.th, self.src = None, "none"
+
+    def mark(self, start):
+        if start:
+            self.t0 = time.perf_counter()
+        else:
+            self.t1 = time.perf_counter()
 
     def stop(self):
-        if self.p is None:
+        if self.th is None:
             return None
-        self.p.terminate()
-        self.p.wait()
-        rows = []
-        for line in open(self.out):
-            f = [x.strip() for x in line.split(",")]
-            if len(f) >= 7:
-                try:
-                    rows.append((float(f[0]), float(f[1]), f[3:7]))
-                except ValueError:
-                    pass
-        if not rows:
+        time.sleep(0.012)      # one more sample after the region closes
+        self._stop.set()
+        self.th.join()
+        rows = self.rows
+        if not rows or self.t0 is None or self.t1 is None:
             return None
-        load = [r for r in rows if r[0] > 500] or rows
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in load for i, v in enumerate(r[2]) if v.lower().startswith("active")})
-        return {"sm_mhz": statistics.median(r[0] for r in load), "sm_max_mhz": max(r[1] for r in rows),
-                "reasons": reasons, "samples": len(load)}
+        inside = [r for r in rows if self.t0 <= r[0] <= self.t1]
+        before = [r for r in rows if r[0] < self.t0][-1:]
+        after = [r for r in rows if r[0] > self.t1][:1]
+        win = before + inside + after if len(inside) < 3 else inside
+        reasons = sorted({nm for r in win for bit, nm in self.REASONS.items() if r[2] & bit})
+        return {"sm_mhz": statistics.median(r[1] for r in win), "sm_max_mhz": self.max_mhz,
+                "sm_min_mhz": min(r[1] for r in win), "reasons": reasons, "samples": len(win),
+                "samples_inside": len(inside), "window_ms": round((self.t1 - self.t0) * 1e3, 3),
+                "source": "nvml 5 ms poll"}
 
 
 # ------------------------------------------------------------------ reference arm (CPU oracle)
@@ -202,6 +243,50 @@ def run_reference(args, wl):
 
 
 # ------------------------------------------------------------------ GPU arm
+def relaunch(args):
+    """`--gpus N` without torchrun: run this script under torch.distributed.run with N local
+    ranks (rendezvous on 127.0.0.1) and exit with its status."""
+    import socket
+    import subprocess
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    env.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    print(f"[bench] launching {args.gpus} ranks: {' '.join(cmd)}", file=sys.stderr, flush=True)
+    sys.exit(subprocess.run(cmd, env=env).returncode)
+
+
+def dry_run(args):
+    """The launch path without GPU work: gloo group, world == --gpus, each rank's strip."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_pitaksirianannt16_b200 as tbs
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    n = WORKLOADS[args.workload][2]
+    if world > 1:
+        dist.init_process_group("gloo")
+    rows = list(tbs.rank_rows(n, world, rank))
+    got = [None] * world
+    if world > 1:
+        dist.all_gather_object(got, (rank, os.getpid(), rows))
+        dist.barrier()
+        dist.destroy_process_group()
+    else:
+        got = [(rank, os.getpid(), rows)]
+    if rank == 0:
+        print(json.dumps({"dry_run": True, "n_gpus": world, "gpus_requested": args.gpus, "workload": args.workload,
+                          "n": n, "combine": args.combine, "impl": args.impl,
+                          "ranks": [{"rank": r, "pid": pid, "rows": rw} for r, pid, rw in got]}), flush=True)
+    del torch
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -211,7 +296,16 @@ def main():
     ap.add_argument("--impl", default="tbs", choices=["tbs", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--combine", default="nccl", choices=["nccl", "fused"],
+                    help="N > 1, SDH / 2PCF: NCCL all_reduce (default) or the fused peer-memory flush")
+    ap.add_argument("--dry-run", action="store_true", help="launch path only (gloo, no GPU work)")
     args = ap.parse_args()
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        return relaunch(args)
+    world_env = int(os.environ.get("WORLD_SIZE", "1"))
+    assert world_env == args.gpus, f"WORLD_SIZE = {world_env} but --gpus {args.gpus}"
+    if args.dry_run:
+        return dry_run(args)
     assert args.warmup >= 3 or args.impl == "reference", "timing rules: >= 3 warm-up steps"
     wl = args.workload
     if args.impl == "reference":
@@ -229,6 +323,8 @@ def main():
     dev = torch.device("cuda", local)
     pg = None
     if world > 1:
+        for k, v in (("NCCL_DEBUG", "INFO"), ("NCCL_DEBUG_SUBSYS", "INIT"), ("NCCL_DEBUG_FILE", "/dev/stderr")):
+            os.environ.setdefault(k, v)      # communicator ranks in the log, stdout kept for the JSON line
         dist.init_process_group("nccl", device_id=dev)
         pg = dist.group.WORLD
 
@@ -256,17 +352,19 @@ def main():
         rows_pm = (n * rank // world, n * (rank + 1) // world)
         out = torch.empty((rows_pm[1] - rows_pm[0], n), dtype=torch.float32, device=dev)
 
-    # N > 1, Type-I/II: the combine is fused into the kernels' flush (every partial is added
-    # into every rank's buffer over NVLink peer memory, TBS_OUT_PEERS); NCCL all_reduce only
-    # if the peer mapping cannot be set up.
+    # N > 1, Type-I/II: one NCCL all_reduce of the per-rank histogram / count (--combine nccl),
+    # or the combine fused into the kernels' flush (every partial added into every rank's buffer
+    # over NVLink peer memory, TBS_OUT_PEERS; --combine fused), falling back to NCCL if the peer
+    # mapping cannot be set up (no native peer atomics, ...). config.combine records what ran.
     sink, combine = None, "none"
     if pg is not None and op in ("sdh", "sdh_lattice", "pcf"):
-        try:
-            sink = tbs.PeerSink(nb if op != "pcf" else 1, pg, dev)
-            combine = "fused-peer"
-        except Exception as e:   # noqa: BLE001 — report and use the collective instead
-            print(f"[bench] fused combine unavailable ({e}); using NCCL all_reduce", file=sys.stderr)
-            combine = "nccl-allreduce"
+        combine = "nccl-allreduce"
+        if args.combine == "fused":
+            try:
+                sink = tbs.PeerSink(nb if op != "pcf" else 1, pg, dev)
+                combine = "fused-peer"
+            except Exception as e:   # noqa: BLE001 — report and use the collective instead
+                print(f"[bench] fused combine unavailable ({e}); using NCCL all_reduce", file=sys.stderr)
     elif pg is not None:
         combine = "nccl-allreduce" if op == "kde" else "none (row-sharded output)"
 
@@ -297,10 +395,12 @@ def main():
     if pg is not None:
         dist.barrier()
     torch.cuda.synchronize(dev)
-    clocks = Clocks(local) if rank == 0 else None
+    clocks = Clocks(dev) if rank == 0 else None
     l0 = tbs.launch_count()
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     sev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    if clocks:
+        clocks.mark(True)
     t0.record(st)
     for k in range(args.steps):
         flush.fill_(k & 0xFF)    # L2 flush between steps (256 MiB > 126 MB L2), outside the step events
@@ -309,6 +409,8 @@ def main():
         sev[k][1].record(st)
     t1.record(st)
     torch.cuda.synchronize(dev)
+    if clocks:
+        clocks.mark(False)
     if pg is not None:
         dist.barrier()
     launches = tbs.launch_count() - l0

@@ -45,8 +45,9 @@
  * zero output. Allocation failure returns TBS_ENOMEM; a CUDA error returns
  * TBS_ECUDA. tbs_last_error() gives a thread-local message for the last non-OK
  * status. Non-finite coordinates are a caller contract violation (not checked on
- * the hot path). Under TBS_EXACT_LATTICE, coordinates must be integer-valued with
- * every squared pair distance < 2^24 (exact in fp32) and 4^j * s < 2^62.
+ * the hot path; TBS_VALIDATE checks them). Under TBS_EXACT_LATTICE, coordinates must be
+ * integer-valued with every squared pair distance < 2^24 (exact in fp32) and 4^j * s < 2^62
+ * (TBS_VALIDATE checks the first two).
  */
 #ifndef TBS_H_
 #define TBS_H_
@@ -80,14 +81,23 @@ typedef struct {
 #define TBS_FORCE_CLAMP 0x100u        /* SDH: never elide the nb-1 clamp (ablation/tests)   */
 #define TBS_HIST_FORCE_PASSES 0x200u  /* SDH: bucket-range passes with one smem copy (tests)   */
 /* SDH / 2PCF: fused multi-GPU combine (the paper's multi-GPU future work,
- * L1254-1256). Instead of writing hist / count, every partial the kernels flush (a9) is added
- * with a system-scope atomic into EACH of args->out_peers[0 .. n_out_peers) — uint64 [nb]
- * (SDH) or [1] (2PCF) device buffers, the local rank's own and the other ranks' mapped over
- * NVLink by CUDA IPC (tbs_peer_open). Nothing is zeroed: the caller zeroes every rank's buffer
- * before any rank's call starts, and after every rank's call has completed each buffer holds
- * the sum over all ranks' row ranges (the all-reduce, without a separate collective).
- * hist / count may be NULL. Other entry points return TBS_EUNSUPPORTED for this flag. */
+ * L1254-1256). Instead of writing hist / count, the call accumulates its (row-range) partial in
+ * a local device buffer and, as its last kernel, adds that partial with system-scope atomics
+ * into EACH of args->out_peers[0 .. n_out_peers) — uint64 [out_peer_words] device buffers,
+ * out_peer_words = nb (SDH) or 1 (2PCF): the local rank's own and the other ranks' mapped over
+ * NVLink by CUDA IPC (tbs_peer_open; peers need native atomics, tbs_peer_atomics_ok). That is
+ * out_peer_words x n_out_peers remote adds per rank. Nothing is zeroed: the caller zeroes
+ * every rank's buffer before any rank's call starts, and after every rank's call has completed
+ * each buffer holds the sum over all ranks' row ranges (the all-reduce, without a separate
+ * collective). hist / count may be NULL. Other entry points return TBS_EUNSUPPORTED. */
 #define TBS_OUT_PEERS 0x400u
+/* Debug validation: the loader's pass over the points also records non-finite
+ * and non-integer coordinates and the bounding box; with TBS_VALIDATE the call waits for it
+ * (one stream synchronisation) and returns TBS_EINVAL, before any pair kernel runs, if a
+ * coordinate is non-finite or, under TBS_EXACT_LATTICE, non-integer or spread so far that a
+ * squared pair distance could reach 2^24 (sum over the coordinates of (max - min)^2 >= 2^24).
+ * Not for the hot path: it costs a host round trip. SDH, 2PCF, kernel density, RDF. */
+#define TBS_VALIDATE 0x800u
 
 #define TBS_MAX_N ((int64_t)1 << 30)
 #define TBS_MAX_BUCKETS (1 << 24)
@@ -116,6 +126,8 @@ typedef struct {
   void* ev_end;         /* optional cudaEvent_t recorded just after it (profiling hook)     */
   void* const* out_peers; /* TBS_OUT_PEERS: device pointers of every rank's output buffer     */
   int n_out_peers;      /* 1 .. TBS_MAX_PEERS                                              */
+  int64_t out_peer_words; /* TBS_OUT_PEERS: uint64 words of EVERY out_peers buffer; must equal
+                             nbuckets (SDH) or 1 (2PCF), else TBS_EINVAL                    */
 } tbs_args;
 #define TBS_MAX_PEERS 16
 
@@ -146,10 +158,23 @@ int tbs_kde_ex(const tbs_args* args, float gamma, double* sum);   /* sum: device
 int tbs_knn(const float* points, int64_t n, int dim, int k, int32_t* idx, float* dist);
 int tbs_knn_ex(const tbs_args* args, int k, int32_t* idx, float* dist);
 
-/* Radial distribution function, "a normalized form of SDH": host arrays,
- * g[k] = hist[k] / (C(n,2) * shell_k / volume), shell_k the dim-ball shell volume between
- * k w and (k+1) w (no periodic boundary). Host-only arithmetic on an SDH result. */
-int tbs_rdf(const uint64_t* hist, int nbuckets, int dim, float bucket_width, int64_t n, double volume, double* g);
+/* Radial distribution function, "a normalized form of SDH" (§III-B; DESIGN.md
+ * reading R6). For the nb real shells k w <= d < (k+1) w, k = 0..nb-1:
+ *   g[k] = h[k] / (P * shell_k / volume),  shell_k = c_dim (((k+1) w)^dim - (k w)^dim),
+ * c_dim the unit dim-ball volume (no periodic boundary), h the SDH of the same pairs computed
+ * with nb+1 buckets (bucket nb holds every d >= nb w and is not a shell, so it is dropped) and
+ * P the number of pairs h counts: sum over the anchor rows i in [row_begin, row_end) of
+ * (n - 1 - i) (C(n,2) for the whole set). g: fp64 [nb], overwritten. TBS_EXACT_LATTICE and the
+ * SDH's other flags apply to the histogram (TBS_OUT_PEERS: TBS_EUNSUPPORTED, use
+ * tbs_rdf_hist_ex on the combined histogram). volume must be finite and > 0.
+ * tbs_rdf: host or device pointers, synchronous. tbs_rdf_ex: device pointers, enqueued. */
+int tbs_rdf(const float* points, int64_t n, int dim, float bucket_width, int nbuckets, double volume, double* g);
+int tbs_rdf_ex(const tbs_args* args, float bucket_width, int nbuckets, double volume, double* g);
+/* The normalisation alone, on the device, for a histogram combined across ranks: hist is a
+ * device uint64 [>= nbuckets] (its first nbuckets real shells are used), pairs the pairs it
+ * counts (n(n-1)/2 after the all-reduce), g a device fp64 [nbuckets]; enqueued on `stream`. */
+int tbs_rdf_hist_ex(const uint64_t* hist, int nbuckets, int dim, float bucket_width, double pairs, double volume,
+                    double* g, void* stream);
 
 /* High-dimensional Type-III pair matrix on the 5th-generation tensor cores (NEXT-3;
  * PAPER.md L330-332 kernel methods over feature spaces): features are bf16 [n][d] row-major
@@ -177,6 +202,12 @@ int tbs_peer_alloc(uint64_t bytes, void** dev_ptr, void* handle);
 int tbs_peer_open(const void* handle, void** dev_ptr);
 int tbs_peer_close(void* dev_ptr);
 int tbs_peer_free(void* dev_ptr);
+/* *ok = 1 if the current device can add into memory of the GPU with PCI bus id `pci_bus_id`
+ * ("dddd:bb:dd.f") with native atomics (same device, or peer access with
+ * cudaDevP2PAttrNativeAtomicSupported); 0 otherwise, including a GPU this process cannot see.
+ * The fused combine relies on system-scope atomics over peer memory: without native support
+ * (e.g. PCIe P2P) the adds are not atomic, so callers must fall back to the all-reduce. */
+int tbs_peer_atomics_ok(const char* pci_bus_id, int* ok);
 
 /* Thread-local text of the last non-OK status ("" if none). */
 const char* tbs_last_error(void);

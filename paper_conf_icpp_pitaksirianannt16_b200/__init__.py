@@ -14,6 +14,7 @@ library or a CUDA device is missing, calls raise.
     kde(points, gamma)                    Type-I kernel-density pair sum      (float64[1])   (NEXT-2)
     knn(points, k)                        Type-I all-point k nearest neighbours (int32, float32 [n, k]) (NEXT-2)
     rdf(points, bucket_width, nb, volume) radial distribution function       (float64[nb])  (NEXT-1)
+    rdf_from_hist(hist, ...)              its normalisation on a (combined) device histogram
     sdh_host / pcf_host / pairmatrix_host the same through host (numpy) buffers
 """
 from __future__ import annotations
@@ -34,6 +35,7 @@ TBS_HIST_FORCE_GLOBAL = 0x40
 TBS_FORCE_CLAMP = 0x100
 TBS_HIST_FORCE_PASSES = 0x200
 TBS_OUT_PEERS = 0x400
+TBS_VALIDATE = 0x800
 TBS_MAX_PEERS = 16
 KERNELS = {"gaussian": 0, "dist2": 1, "dist": 2}
 HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "global": TBS_HIST_FORCE_GLOBAL,
@@ -41,8 +43,9 @@ HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "
 
 # Symbols declared in include/tbs.h (checked by tests/test_abi.py).
 EXPORTS = ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
-           "tbs_kde", "tbs_kde_ex", "tbs_knn", "tbs_knn_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex",
-           "tbs_rank_rows", "tbs_peer_alloc", "tbs_peer_open", "tbs_peer_close", "tbs_peer_free",
+           "tbs_kde", "tbs_kde_ex", "tbs_knn", "tbs_knn_ex", "tbs_rdf", "tbs_rdf_ex", "tbs_rdf_hist_ex",
+           "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex",
+           "tbs_rank_rows", "tbs_peer_alloc", "tbs_peer_open", "tbs_peer_close", "tbs_peer_free", "tbs_peer_atomics_ok",
            "tbs_last_error", "tbs_release", "tbs_launch_count", "tbs_version")
 
 
@@ -54,7 +57,8 @@ class _Args(ctypes.Structure):
     _fields_ = [("points", ctypes.c_void_p), ("n", ctypes.c_int64), ("dim", ctypes.c_int),
                 ("row_begin", ctypes.c_int64), ("row_end", ctypes.c_int64), ("stream", ctypes.c_void_p),
                 ("flags", ctypes.c_uint32), ("ev_begin", ctypes.c_void_p), ("ev_end", ctypes.c_void_p),
-                ("out_peers", ctypes.POINTER(ctypes.c_void_p)), ("n_out_peers", ctypes.c_int)]
+                ("out_peers", ctypes.POINTER(ctypes.c_void_p)), ("n_out_peers", ctypes.c_int),
+                ("out_peer_words", ctypes.c_int64)]
 
 
 class _Kernel(ctypes.Structure):
@@ -82,7 +86,11 @@ def lib() -> ctypes.CDLL:
         L.tbs_kde_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_float, vp]
         L.tbs_knn.argtypes = [vp, i64, ctypes.c_int, ctypes.c_int, vp, vp]
         L.tbs_knn_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_int, vp, vp]
-        L.tbs_rdf.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_float, i64, ctypes.c_double, vp]
+        L.tbs_rdf.argtypes = [vp, i64, ctypes.c_int, ctypes.c_float, ctypes.c_int, ctypes.c_double, vp]
+        L.tbs_rdf_ex.argtypes = [ctypes.POINTER(_Args), ctypes.c_float, ctypes.c_int, ctypes.c_double, vp]
+        L.tbs_rdf_hist_ex.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_float, ctypes.c_double, ctypes.c_double,
+                                      vp, vp]
+        L.tbs_peer_atomics_ok.argtypes = [ctypes.c_char_p, ctypes.POINTER(ctypes.c_int)]
         L.tbs_pairmatrix_hd.argtypes = [vp, i64, ctypes.c_int, _Kernel, vp]
         L.tbs_pairmatrix_hd_ex.argtypes = [vp, i64, ctypes.c_int, i64, i64, _Kernel, vp, vp, vp, vp]
         L.tbs_rank_rows.argtypes = [i64, ctypes.c_int, ctypes.c_int, ctypes.POINTER(ctypes.c_int64),
@@ -95,8 +103,9 @@ def lib() -> ctypes.CDLL:
         L.tbs_launch_count.restype = ctypes.c_uint64
         L.tbs_release.restype = None
         for f in ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",
-                  "tbs_kde", "tbs_kde_ex", "tbs_knn", "tbs_knn_ex", "tbs_rdf", "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex", "tbs_rank_rows", "tbs_version",
-                  "tbs_peer_alloc", "tbs_peer_open", "tbs_peer_close", "tbs_peer_free"):
+                  "tbs_kde", "tbs_kde_ex", "tbs_knn", "tbs_knn_ex", "tbs_rdf", "tbs_rdf_ex", "tbs_rdf_hist_ex",
+                  "tbs_pairmatrix_hd", "tbs_pairmatrix_hd_ex", "tbs_rank_rows", "tbs_version",
+                  "tbs_peer_alloc", "tbs_peer_open", "tbs_peer_close", "tbs_peer_free", "tbs_peer_atomics_ok"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -142,10 +151,11 @@ def partition(n: int, group=None, rows=None):
 
 class PeerSink:
     """Buffers of the fused combine (TBS_OUT_PEERS): one int64[words] device buffer per rank
-    of `group`, each mapped into every rank (CUDA IPC; over NVLink between GPUs). A call
-    with ``sink=`` adds every partial its kernels flush into all of them, so after
-    ``finish()`` each rank's buffer holds the all-reduced result — the collective is fused
-    into the kernels' flush instead of a separate NCCL all_reduce.
+    of `group`, each mapped into every rank (CUDA IPC; over NVLink between GPUs; every peer
+    must be reachable with native atomics). A call with ``sink=`` accumulates its row strip's
+    partial locally and its last kernel adds it into all of them (system-scope atomics: words x
+    ranks remote adds per rank), so after ``finish()`` each rank's buffer holds the all-reduced
+    result — the collective is fused into the call instead of a separate NCCL all_reduce.
 
     Every rank holds two buffers (parity p = result index & 1), so one host barrier per
     result suffices: ``begin(stream)`` enqueues the zeroing of this rank's OTHER-parity buffer
@@ -174,11 +184,20 @@ class PeerSink:
             else:
                 err = "tbs_peer_alloc: " + last_error()
             handles = [None] * self.world
-            mine = h.raw if self._own is not None else None
+            pr = torch.cuda.get_device_properties(dev)
+            bus = f"{pr.pci_domain_id:04x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+            mine = (h.raw, bus) if self._own is not None else None
             if group is not None:
                 dist.all_gather_object(handles, mine, group=group)
             else:
                 handles[0] = mine
+            # the fused adds are system-scope atomics into peer memory: every peer GPU must be
+            # reachable with NATIVE atomics (NVLink; not PCIe P2P), else all ranks fall back
+            for r, hr in enumerate(handles):
+                if hr is not None and err is None:
+                    okp = ctypes.c_int(0)
+                    if lib().tbs_peer_atomics_ok(hr[1].encode(), ctypes.byref(okp)) != TBS_OK or not okp.value:
+                        err = f"no native peer atomics to rank {r} (GPU {hr[1]})"
             ptrs = []
             for r, hr in enumerate(handles):
                 if r == self.rank:
@@ -188,7 +207,7 @@ class PeerSink:
                     ptrs.append(None)
                 else:
                     q = ctypes.c_void_p()
-                    if lib().tbs_peer_open(hr, ctypes.byref(q)) == TBS_OK:
+                    if lib().tbs_peer_open(hr[0], ctypes.byref(q)) == TBS_OK:
                         self._opened.append(q.value)
                         ptrs.append(q.value)
                     else:
@@ -260,7 +279,7 @@ class _CudaArray:
 def _fused(a, sink):
     if sink is not None:
         a.flags |= TBS_OUT_PEERS
-        a.out_peers, a.n_out_peers = sink.ptrs, sink.world
+        a.out_peers, a.n_out_peers, a.out_peer_words = sink.ptrs, sink.world, sink.words
     return a
 
 
@@ -291,14 +310,15 @@ def _args(points, rows, flags, stream, events):
     n, dim = points.shape
     rb, re = (0, n) if rows is None else (int(rows[0]), int(rows[1]))
     st = stream if stream is not None else torch.cuda.current_stream(points.device)
-    a = _Args(points.data_ptr(), n, dim, rb, re, st.cuda_stream, flags, None, None)
+    a = _Args(points.data_ptr(), n, dim, rb, re, st.cuda_stream, flags, None, None, None, 0, 0)
     if events is not None:
         a.ev_begin, a.ev_end = events[0].cuda_event, events[1].cuda_event
     return a, n
 
 
 def sdh(points, bucket_width: float, nbuckets: int, *, rows=None, lattice: bool = False, hist_mode=None,
-        force_clamp: bool = False, out=None, stream=None, events=None, group=None, sink=None):
+        force_clamp: bool = False, validate: bool = False, out=None, stream=None, events=None, group=None,
+        sink=None):
     """Spatial distance histogram (Type-II). Returns int64[nbuckets] on points.device.
 
     rows=(b, e): only anchors i in [b, e) (with all partners j > i). lattice=True:
@@ -306,11 +326,16 @@ def sdh(points, bucket_width: float, nbuckets: int, *, rows=None, lattice: bool 
     group: a torch.distributed process group: each rank computes its pair-balanced
     strip (rank_rows) and the partial histograms are summed with one all_reduce, or, with
     sink=PeerSink(nbuckets, group), by the kernels' own flush into every rank's buffer.
+    validate=True: TBS_VALIDATE (debug; raises on non-finite coordinates and, with lattice, on a
+    violated exact-lattice contract).
     """
     torch = _torch()
-    flags = (TBS_EXACT_LATTICE if lattice else 0) | HIST_MODES[hist_mode] | (TBS_FORCE_CLAMP if force_clamp else 0)
+    flags = (TBS_EXACT_LATTICE if lattice else 0) | HIST_MODES[hist_mode] | (TBS_FORCE_CLAMP if force_clamp else 0) \
+        | (TBS_VALIDATE if validate else 0)
     a, _ = _args(points, partition(points.shape[0], group, rows), flags, stream, events)
     if sink is not None:            # fused combine: the kernels' flush is the all-reduce
+        if sink.words != nbuckets:
+            raise ValueError(f"sink holds {sink.words} words, the histogram has {nbuckets}")
         sink.begin(stream)
         _check(lib().tbs_sdh_ex(ctypes.byref(_fused(a, sink)), float(bucket_width), int(nbuckets), None), "tbs_sdh_ex")
         return sink.finish(stream, out)
@@ -319,12 +344,15 @@ def sdh(points, bucket_width: float, nbuckets: int, *, rows=None, lattice: bool 
     return combine(h, group)
 
 
-def pcf(points, radius: float, *, rows=None, out=None, stream=None, events=None, group=None, sink=None):
+def pcf(points, radius: float, *, rows=None, validate: bool = False, out=None, stream=None, events=None, group=None,
+        sink=None):
     """2-point correlation count (Type-I): #{i<j : d < radius}, int64[1] on points.device.
     sink=PeerSink(1, group): fused combine (see sdh)."""
     torch = _torch()
-    a, _ = _args(points, partition(points.shape[0], group, rows), 0, stream, events)
+    a, _ = _args(points, partition(points.shape[0], group, rows), TBS_VALIDATE if validate else 0, stream, events)
     if sink is not None:
+        if sink.words != 1:
+            raise ValueError(f"sink holds {sink.words} words, the 2PCF count has 1")
         sink.begin(stream)
         _check(lib().tbs_pcf_ex(ctypes.byref(_fused(a, sink)), float(radius), None), "tbs_pcf_ex")
         return sink.finish(stream, out)
@@ -365,19 +393,41 @@ def knn(points, k: int, *, rows=None, out=None, stream=None, events=None, group=
     return idx, dist_
 
 
-def rdf_from_hist(hist, bucket_width: float, n: int, volume: float, dim: int = 3):
-    """RDF g[k] (NEXT-1) from an SDH histogram (host arithmetic in libtbs: tbs_rdf)."""
-    h = np.ascontiguousarray(hist.cpu().numpy() if hasattr(hist, "cpu") else hist).astype(np.uint64)
-    gr = np.empty(len(h), np.float64)
-    _check(lib().tbs_rdf(h.ctypes.data, len(h), int(dim), float(bucket_width), int(n), float(volume), gr.ctypes.data),
-           "tbs_rdf")
-    return gr
+def rdf_from_hist(hist, bucket_width: float, nbuckets: int, volume: float, pairs: int, dim: int = 3, *, out=None,
+                  stream=None):
+    """RDF normalisation (NEXT-1, reading R6) of a device int64 histogram of >= nbuckets shells
+    (e.g. an SDH with nbuckets + 1 buckets combined across ranks) counting `pairs` pairs; runs on
+    the device (tbs_rdf_hist_ex). Returns float64[nbuckets] on the histogram's device."""
+    torch = _torch()
+    if not (isinstance(hist, torch.Tensor) and hist.is_cuda and hist.dtype == torch.int64 and hist.numel() >= nbuckets):
+        raise TypeError("hist must be a CUDA int64 tensor with >= nbuckets entries")
+    st = stream if stream is not None else torch.cuda.current_stream(hist.device)
+    g = out if out is not None else torch.empty(nbuckets, dtype=torch.float64, device=hist.device)
+    _check(lib().tbs_rdf_hist_ex(hist.contiguous().data_ptr(), int(nbuckets), int(dim), float(bucket_width),
+                                 float(pairs), float(volume), g.data_ptr(), st.cuda_stream), "tbs_rdf_hist_ex")
+    return g
 
 
-def rdf(points, bucket_width: float, nbuckets: int, volume: float, **kw):
-    """Radial distribution function: SDH on the GPU, then the ideal-gas normalisation."""
-    h = sdh(points, bucket_width, nbuckets, **kw)
-    return rdf_from_hist(h, bucket_width, points.shape[0], volume, points.shape[1] if points.dim() > 1 else 1)
+def rdf(points, bucket_width: float, nbuckets: int, volume: float, *, rows=None, lattice: bool = False,
+        hist_mode=None, validate: bool = False, out=None, stream=None, events=None, group=None, sink=None):
+    """Radial distribution function g[k], k < nbuckets (NEXT-1, reading R6): the SDH of the same
+    pairs with nbuckets + 1 buckets (the clamp bucket is dropped), normalised on the device by
+    the ideal-gas shell counts of the pairs counted (tbs_rdf_ex). With a group, the ranks' SDH
+    strips are combined first (all_reduce, or sink=PeerSink(nbuckets + 1, group)) and the
+    normalisation uses all n(n-1)/2 pairs."""
+    torch = _torch()
+    n = points.shape[0]
+    dim = points.shape[1] if points.dim() > 1 else 1
+    if group is not None:
+        h = sdh(points, bucket_width, nbuckets + 1, lattice=lattice, hist_mode=hist_mode, stream=stream,
+                events=events, group=group, sink=sink)
+        return rdf_from_hist(h, bucket_width, nbuckets, volume, n * (n - 1) // 2, dim, out=out, stream=stream)
+    flags = (TBS_EXACT_LATTICE if lattice else 0) | HIST_MODES[hist_mode] | (TBS_VALIDATE if validate else 0)
+    a, _ = _args(points, rows, flags, stream, events)
+    g = out if out is not None else torch.empty(nbuckets, dtype=torch.float64, device=points.device)
+    _check(lib().tbs_rdf_ex(ctypes.byref(a), float(bucket_width), int(nbuckets), float(volume), g.data_ptr()),
+           "tbs_rdf_ex")
+    return g
 
 
 def pairmatrix(points, gamma: float = 1.0, *, kernel: str = "gaussian", rows=None, out=None, stream=None,

@@ -20,6 +20,7 @@
 #include "tbs_hd.cuh"
 #include "tbs_hd2.cuh"
 #include "tbs_knn.cuh"
+#include "tbs_rdf.cuh"
 
 using namespace tbs;
 static_assert(kMaxPeers == TBS_MAX_PEERS, "peer sink size");
@@ -221,14 +222,19 @@ int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op
   return TBS_OK;
 }
 
-int validate_common(const tbs_args* a, bool peers_ok = false) {
+// peer_words: the output words of this operation (SDH nb, 2PCF 1) under TBS_OUT_PEERS; 0 = the
+// operation does not support the fused combine.
+int validate_common(const tbs_args* a, long long peer_words = 0) {
   if (!a) return fail(TBS_EINVAL, "args is NULL");
   if (a->flags & TBS_OUT_PEERS) {
-    if (!peers_ok) return fail(TBS_EUNSUPPORTED, "TBS_OUT_PEERS: SDH and 2PCF only");
+    if (peer_words == 0) return fail(TBS_EUNSUPPORTED, "TBS_OUT_PEERS: SDH and 2PCF only");
     if (a->n_out_peers < 1 || a->n_out_peers > kMaxPeers || !a->out_peers)
       return fail(TBS_EINVAL, "TBS_OUT_PEERS needs 1..%d out_peers", kMaxPeers);
     for (int w = 0; w < a->n_out_peers; ++w)
       if (!a->out_peers[w]) return fail(TBS_EINVAL, "out_peers[%d] is NULL", w);
+    if (a->out_peer_words != peer_words)
+      return fail(TBS_EINVAL, "TBS_OUT_PEERS: out_peer_words = %lld, this call writes %lld words",
+                  (long long)a->out_peer_words, peer_words);
   }
   if (a->n < 0 || a->n > TBS_MAX_N) return fail(TBS_EINVAL, "n = %lld outside [0, 2^30]", (long long)a->n);
   if (a->dim < 1 || a->dim > 4) return fail(TBS_EINVAL, "dim = %d outside [1, 4]", a->dim);
@@ -246,9 +252,12 @@ int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long 
   const size_t soa_bytes = (size_t)D * n_pad * sizeof(float);
   TBS_CUDA(cudaMallocAsync((void**)soa, soa_bytes + 64, st));
   *bbox = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(*soa) + soa_bytes);
-  TBS_CUDA(cudaMemsetAsync(*bbox, 0, 64, st));
-  const int threads = 256;
-  long long blocks = std::min<long long>((n_pad + threads - 1) / threads, 148ll * 16);
+  // Small problems: one 1024-thread CTA writes the whole bounding-box block itself (no memset
+  // launch before it: the small-problem path is latency-bound, BASELINE configs[0]).
+  const bool one = n_pad <= 16384 && zero_words <= (1 << 16);
+  if (!one) TBS_CUDA(cudaMemsetAsync(*bbox, 0, 64, st));
+  const int threads = one ? 1024 : 256;
+  long long blocks = one ? 1 : std::min<long long>((n_pad + threads - 1) / threads, 148ll * 16);
   blocks = std::max<long long>(blocks, 1);
   soa_loader<<<(unsigned)blocks, threads, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, D, pad, *soa, zero,
                                                    zero_words, *bbox);
@@ -257,17 +266,53 @@ int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long 
   return TBS_OK;
 }
 
-// Output sink of a Type-I/II call: the caller's buffer, or every rank's (TBS_OUT_PEERS).
-OutSink make_sink(const tbs_args* a, unsigned long long* own) {
-  OutSink o{};
-  if (a->flags & TBS_OUT_PEERS) {
-    o.n = a->n_out_peers;
-    for (int w = 0; w < o.n; ++w) o.p[w] = reinterpret_cast<unsigned long long*>(a->out_peers[w]);
-  } else {
-    o.n = 0;
-    o.p[0] = own;
+// TBS_VALIDATE (debug): wait for the loader and check what it recorded in the
+// bounding-box block: non-finite coordinates; under the exact-lattice contract also non-integer
+// coordinates and a spread whose squared pair distances could reach 2^24.
+int validate_points(const tbs_args* a, const uint32_t* bbox, int D, bool lattice, cudaStream_t st) {
+  if (!(a->flags & TBS_VALIDATE) || a->n < 1) return TBS_OK;
+  uint32_t h[9] = {0};
+  TBS_CUDA(cudaMemcpyAsync(h, bbox, (size_t)(2 * D + 1) * 4, cudaMemcpyDeviceToHost, st));
+  TBS_CUDA(cudaStreamSynchronize(st));
+  if (h[2 * D] & 1u) return fail(TBS_EINVAL, "TBS_VALIDATE: non-finite coordinate");
+  if (lattice) {
+    if (h[2 * D] & 2u) return fail(TBS_EINVAL, "TBS_VALIDATE: TBS_EXACT_LATTICE needs integer-valued coordinates");
+    auto ord2f_h = [](uint32_t o) {
+      const uint32_t b = (o & 0x80000000u) ? (o & 0x7fffffffu) : ~o;
+      float f;
+      memcpy(&f, &b, 4);
+      return (double)f;
+    };
+    double s = 0.0;
+    for (int c = 0; c < D; ++c) {
+      const double e = ord2f_h(h[D + c]) - ord2f_h(~h[c]);
+      s += e * e;
+    }
+    if (s >= 16777216.0)
+      return fail(TBS_EINVAL, "TBS_VALIDATE: TBS_EXACT_LATTICE needs every squared pair distance < 2^24 "
+                  "(bounding-box bound %.0f)", s);
   }
+  return TBS_OK;
+}
+
+// Output sink of the kernels of a Type-I/II call: one device buffer (the caller's output, or
+// under TBS_OUT_PEERS the call's local accumulator).
+OutSink local_sink(unsigned long long* buf) {
+  OutSink o{};
+  o.n = 0;
+  o.p[0] = buf;
   return o;
+}
+
+// TBS_OUT_PEERS, second stage: add the local accumulator into every rank's buffer.
+int push_to_peers(const tbs_args* a, const unsigned long long* acc, int words, cudaStream_t st) {
+  OutSink o{};
+  o.n = a->n_out_peers;
+  for (int w = 0; w < o.n; ++w) o.p[w] = reinterpret_cast<unsigned long long*>(a->out_peers[w]);
+  push_peers<<<(words + 255) / 256, 256, 0, st>>>(acc, words, o);
+  TBS_CUDA(cudaGetLastError());
+  g_launches.fetch_add(1);
+  return TBS_OK;
 }
 
 // Decompose a dyadic width w = m * 2^-j (m odd or j = 0). Returns false if not dyadic.
@@ -397,7 +442,7 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
 }
 
 int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
-  int rc = validate_common(a, true);
+  int rc = validate_common(a, nb);
   if (rc) return rc;
   if (nb < 1 || nb > TBS_MAX_BUCKETS) return fail(TBS_EINVAL, "nbuckets = %d outside [1, 2^24]", nb);
   if (!(w > 0.f) || !std::isfinite(w)) return fail(TBS_EINVAL, "bucket_width must be finite and > 0");
@@ -418,7 +463,12 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
     if (!peers) TBS_CUDA(cudaMemsetAsync(h, 0, (size_t)nb * 8, st));   // (fused combine: adds nothing)
     return TBS_OK;
   }
-  const OutSink sink = make_sink(a, h);
+  unsigned long long* acc = nullptr;   // TBS_OUT_PEERS: this rank's partial, pushed to every rank at the end
+  if (peers) {
+    TBS_CUDA(cudaMallocAsync((void**)&acc, (size_t)nb * 8, st));
+    h = acc;
+  }
+  const OutSink sink = local_sink(h);
   // Output-stage plan: lane-private copies (R = 32) while they fit a 96 KB budget (two CTAs
   // per SM), then 4 replicas, then one copy per CTA; beyond that, global partial copies.
   SdhPlan pl{lattice, false, 5};
@@ -475,11 +525,11 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
     zero_words = (long long)G * nb;
   }
   float* soa = nullptr;
-  // Smem modes accumulate into hist: the loader zeroes it. Global mode zeroes the partials
-  // (the reduce kernel overwrites hist). Fused combine: the callers zeroed every rank's buffer.
+  // Smem modes accumulate into hist (or the fused combine's local accumulator): the loader
+  // zeroes it. Global mode zeroes the partials (the reduce kernel overwrites hist).
   uint32_t* bbox = nullptr;
-  rc = load_points(a, D, n_pad, &soa, pl.global ? part : (peers ? nullptr : h), pl.global ? zero_words : (peers ? 0 : nb),
-                   st, &bbox);
+  rc = load_points(a, D, n_pad, &soa, pl.global ? part : h, pl.global ? zero_words : nb, st, &bbox);
+  if (!rc) rc = validate_points(a, bbox, D, lattice, st);
   if (a->flags & TBS_FORCE_CLAMP) bbox = nullptr;
   if (!rc) {
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
@@ -488,13 +538,15 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
     else rc = lattice ? sdh_dispatch<4, true>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee)
                       : sdh_dispatch<4, false>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee);
   }
+  if (!rc && peers) rc = push_to_peers(a, acc, nb, st);
   if (soa) cudaFreeAsync(soa, st);
   if (part) cudaFreeAsync(part, st);
+  if (acc) cudaFreeAsync(acc, st);
   return rc;
 }
 
 int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
-  int rc = validate_common(a, true);
+  int rc = validate_common(a, 1);
   if (rc) return rc;
   if (!(r >= 0.f) || std::isinf(r)) return fail(TBS_EINVAL, "radius must be finite and >= 0");
   const bool peers = (a->flags & TBS_OUT_PEERS) != 0;
@@ -511,10 +563,14 @@ int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
   float* soa = nullptr;
   uint32_t* bbox = nullptr;
   rc = load_points(a, D, pad_rows(a->n), &soa, peers ? nullptr : c, peers ? 0 : 1, st, &bbox);
+  if (!rc) rc = validate_points(a, bbox, D, false, st);
+  // TBS_OUT_PEERS: the local accumulator is the zeroed spare u64 at byte 40 of the bounding-box
+  // block (words 0..2D are the box, 14-15 the work counter)
+  unsigned long long* acc = peers ? reinterpret_cast<unsigned long long*>(bbox + 10) : c;
   if (!rc) {
     PcfOp op{};
     op.r2 = (float)((double)r * (double)r);
-    const OutSink sink = make_sink(a, c);
+    const OutSink sink = local_sink(acc);
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
     const bool small =
         make_geom(a->n, a->row_begin, a->row_end, PcfCfg::TA, PcfCfg::TP).items < (long long)small_items_per_sm() * dev.sms;
@@ -525,6 +581,7 @@ int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
       rc = D == 3 ? launch_pair<PcfOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink)
                   : launch_pair<PcfOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink);
   }
+  if (!rc && peers) rc = push_to_peers(a, acc, 1, st);
   if (soa) cudaFreeAsync(soa, st);
   return rc;
 }
@@ -545,6 +602,7 @@ int kde_impl(const tbs_args* a, float gamma, double* sum) {
   float* soa = nullptr;
   uint32_t* bbox = nullptr;
   rc = load_points(a, D, pad_rows(a->n), &soa, reinterpret_cast<unsigned long long*>(sum), 1, st, &bbox);
+  if (!rc) rc = validate_points(a, bbox, D, false, st);
   if (!rc) {
     KdeOp op{};
     op.c = (float)(-(double)gamma * 1.4426950408889634);
@@ -560,6 +618,44 @@ int kde_impl(const tbs_args* a, float gamma, double* sum) {
                   : launch_pair<KdeOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee);
   }
   if (soa) cudaFreeAsync(soa, st);
+  return rc;
+}
+
+// ---- NEXT-1: radial distribution function (reading R6) ------------------------------------
+int rdf_normalize(const uint64_t* hist, int nb, int dim, float w, double pairs, double volume, double* g,
+                  cudaStream_t st) {
+  const int threads = 256;
+  const int blocks = std::min((nb + threads - 1) / threads, 1024);
+  rdf_kernel<<<blocks, threads, 0, st>>>(reinterpret_cast<const unsigned long long*>(hist), nb, dim, (double)w, pairs,
+                                         volume, g);
+  TBS_CUDA(cudaGetLastError());
+  g_launches.fetch_add(1);
+  return TBS_OK;
+}
+
+int rdf_args_ok(int nb, int dim, float w, double volume, const double* g) {
+  if (nb < 1 || nb >= TBS_MAX_BUCKETS) return fail(TBS_EINVAL, "nbuckets = %d outside [1, 2^24)", nb);
+  if (dim < 1 || dim > 4) return fail(TBS_EINVAL, "dim = %d outside [1, 4]", dim);
+  if (!(w > 0.f) || !std::isfinite(w)) return fail(TBS_EINVAL, "bucket_width must be finite and > 0");
+  if (!(volume > 0.0) || !std::isfinite(volume)) return fail(TBS_EINVAL, "volume must be finite and > 0");
+  if (!g) return fail(TBS_EINVAL, "g is NULL");
+  return TBS_OK;
+}
+
+int rdf_impl(const tbs_args* a, float w, int nb, double volume, double* g) {
+  int rc = validate_common(a);
+  if (rc) return rc;
+  if ((rc = rdf_args_ok(nb, a->dim, w, volume, g))) return rc;
+  cudaStream_t st = (cudaStream_t)a->stream;
+  uint64_t* h = nullptr;
+  TBS_CUDA(cudaMallocAsync((void**)&h, (size_t)(nb + 1) * 8, st));
+  rc = sdh_impl(a, w, nb + 1, h);   // bucket nb takes every d >= nb w (the clamp): not a shell
+  if (!rc) {
+    const double rows = (double)(a->row_end - a->row_begin);
+    const double pairs = rows * (double)(2 * a->n - a->row_begin - a->row_end - 1) / 2.0;
+    rc = rdf_normalize(h, nb, a->dim, w, pairs, volume, g, st);
+  }
+  cudaFreeAsync(h, st);
   return rc;
 }
 
@@ -804,8 +900,9 @@ int knn_impl(const tbs_args* a, int k, int32_t* idx, float* dist) {
 }
 
 // ---- host-or-device simple entry points ------------------------------------------
-int is_device_ptr(const void* p, bool& dev) {
-  dev = false;
+// Where a pointer lives: 0 pageable host, 1 page-locked (pinned) host, 2 device / managed.
+int pointer_kind(const void* p, int& kind) {
+  kind = 0;
   if (!p) return TBS_OK;
   cudaPointerAttributes at;
   cudaError_t e = cudaPointerGetAttributes(&at, p);
@@ -813,7 +910,39 @@ int is_device_ptr(const void* p, bool& dev) {
     cudaGetLastError();
     return TBS_OK;  // unregistered host memory
   }
-  dev = at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+  kind = (at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged) ? 2
+         : at.type == cudaMemoryTypeHost ? 1 : 0;
+  return TBS_OK;
+}
+int is_device_ptr(const void* p, bool& dev) {
+  int k = 0;
+  const int rc = pointer_kind(p, k);
+  dev = k == 2;
+  return rc;
+}
+
+// Per-thread page-locked staging for pageable host buffers of the simple entry points (a copy
+// from pageable memory is staged by the driver synchronously, chunk by chunk; a memcpy into a
+// cached pinned buffer plus one DMA is faster for the small calls this path serves).
+struct Staging {
+  void* p = nullptr;
+  size_t bytes = 0;
+  ~Staging() { if (p) cudaFreeHost(p); }
+};
+int staging(size_t bytes, void** out) {
+  static thread_local Staging s;
+  if (s.bytes < bytes) {
+    if (s.p) cudaFreeHost(s.p);
+    s.p = nullptr;
+    s.bytes = 0;
+    const size_t want = std::max<size_t>(bytes, 1 << 20);
+    if (cudaHostAlloc(&s.p, want, cudaHostAllocDefault) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(TBS_ENOMEM, "cudaHostAlloc(%zu) for host staging failed", want);
+    }
+    s.bytes = want;
+  }
+  *out = s.p;
   return TBS_OK;
 }
 
@@ -824,11 +953,11 @@ int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_b
   if (dim < 1 || dim > 4) return fail(TBS_EINVAL, "dim out of range");
   if (!outp) return fail(TBS_EINVAL, "output is NULL");
   if (n >= 2 && !points) return fail(TBS_EINVAL, "points is NULL");
-  bool pdev = false, odev = false;
-  int rc = is_device_ptr(points, pdev);
-  if (!rc) rc = is_device_ptr(outp, odev);
+  int pk = 0, ok = 0;
+  int rc = pointer_kind(points, pk);
+  if (!rc) rc = pointer_kind(outp, ok);
   if (rc) return rc;
-  if (points && pdev != odev) return fail(TBS_EINVAL, "points and output must both be host or both device pointers");
+  if (points && (pk == 2) != (ok == 2)) return fail(TBS_EINVAL, "points and output must both be host or both device pointers");
   cudaStream_t st = cudaStreamPerThread;
   tbs_args a{};
   a.n = n;
@@ -836,32 +965,47 @@ int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_b
   a.row_begin = 0;
   a.row_end = n;
   a.stream = st;
-  if (odev) {
+  if (ok == 2) {
     a.points = points;
     rc = fn(&a, outp);
     if (!rc) TBS_CUDA(cudaStreamSynchronize(st));
     return rc;
   }
-  float* dp = nullptr;
-  void* dout = nullptr;
   const size_t pbytes = (size_t)n * dim * sizeof(float);
-  if (pbytes) TBS_CUDA(cudaMallocAsync((void**)&dp, pbytes, st));
-  cudaError_t e = cudaMallocAsync(&dout, out_bytes, st);
-  if (e != cudaSuccess) {
-    if (dp) cudaFreeAsync(dp, st);
-    return fail(TBS_ENOMEM, "cudaMallocAsync(%zu): %s", out_bytes, cudaGetErrorString(e));
+  // pageable buffers go through the pinned staging area: [points | output]
+  size_t pin_in = pk == 1 ? 0 : (pbytes + 255) / 256 * 256;
+  size_t pin_out = ok == 1 ? 0 : out_bytes;
+  if (pin_in + pin_out > ((size_t)64 << 20)) pin_in = pin_out = 0;   // large: the driver's own staging
+  unsigned char* stage = nullptr;
+  if (pin_in + pin_out) {
+    void* sp = nullptr;
+    if ((rc = staging(pin_in + pin_out, &sp))) return rc;
+    stage = static_cast<unsigned char*>(sp);
   }
-  if (pbytes) e = cudaMemcpyAsync(dp, points, pbytes, cudaMemcpyHostToDevice, st);
+  const void* src = points;
+  if (pin_in && pbytes) {
+    memcpy(stage, points, pbytes);
+    src = stage;
+  }
+  void* dst_host = pin_out ? static_cast<void*>(stage + pin_in) : outp;
+  // one device allocation: [points | output]
+  const size_t dp_bytes = (pbytes + 255) / 256 * 256;
+  unsigned char* dbuf = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&dbuf, dp_bytes + std::max<size_t>(out_bytes, 4), st);
+  if (e != cudaSuccess) return fail(TBS_ENOMEM, "cudaMallocAsync(%zu): %s", dp_bytes + out_bytes, cudaGetErrorString(e));
+  float* dp = reinterpret_cast<float*>(dbuf);
+  void* dout = dbuf + dp_bytes;
+  if (pbytes) e = cudaMemcpyAsync(dp, src, pbytes, cudaMemcpyHostToDevice, st);
   a.points = dp;
   rc = e != cudaSuccess ? fail(TBS_ECUDA, "H2D copy: %s", cudaGetErrorString(e)) : fn(&a, dout);
   if (!rc) {
-    e = cudaMemcpyAsync(outp, dout, out_bytes, cudaMemcpyDeviceToHost, st);
+    e = cudaMemcpyAsync(dst_host, dout, out_bytes, cudaMemcpyDeviceToHost, st);
     if (e != cudaSuccess) rc = fail(TBS_ECUDA, "D2H copy: %s", cudaGetErrorString(e));
   }
-  if (dp) cudaFreeAsync(dp, st);
-  cudaFreeAsync(dout, st);
+  cudaFreeAsync(dbuf, st);
   e = cudaStreamSynchronize(st);
   if (!rc && e != cudaSuccess) rc = fail(TBS_ECUDA, "sync: %s", cudaGetErrorString(e));
+  if (!rc && pin_out) memcpy(outp, dst_host, out_bytes);
   return rc;
 }
 
@@ -914,20 +1058,27 @@ int tbs_kde(const float* points, int64_t n, float gamma, double* sum) {
   return run_simple(points, n, 3, sum, 8, [&](tbs_args* a, void* out) { return kde_impl(a, gamma, (double*)out); });
 }
 
-int tbs_rdf(const uint64_t* hist, int nbuckets, int dim, float bucket_width, int64_t n, double volume, double* g) {
+int tbs_rdf_ex(const tbs_args* args, float bucket_width, int nbuckets, double volume, double* g) {
   g_err.clear();
-  if (!hist || !g || nbuckets < 1 || dim < 1 || dim > 4 || !(bucket_width > 0.f) || !std::isfinite(bucket_width) ||
-      !(volume > 0.0) || !std::isfinite(volume) || n < 0)
-    return fail(TBS_EINVAL, "tbs_rdf: bad arguments");
-  static const double unit_ball[5] = {0.0, 2.0, 3.14159265358979323846, 4.18879020478639098462,
-                                      4.93480220054467930942};
-  const double w = (double)bucket_width, pairs = (double)n * (double)(n - 1) / 2.0;
-  for (int k = 0; k < nbuckets; ++k) {
-    const double shell = unit_ball[dim] * (std::pow((k + 1) * w, dim) - std::pow(k * w, dim));
-    const double ideal = pairs * shell / volume;
-    g[k] = ideal > 0.0 ? (double)hist[k] / ideal : 0.0;
-  }
-  return TBS_OK;
+  return rdf_impl(args, bucket_width, nbuckets, volume, g);
+}
+
+int tbs_rdf_hist_ex(const uint64_t* hist, int nbuckets, int dim, float bucket_width, double pairs, double volume,
+                    double* g, void* stream) {
+  g_err.clear();
+  int rc = rdf_args_ok(nbuckets, dim, bucket_width, volume, g);
+  if (rc) return rc;
+  if (!hist) return fail(TBS_EINVAL, "hist is NULL");
+  if (!(pairs >= 0.0) || !std::isfinite(pairs)) return fail(TBS_EINVAL, "pairs must be finite and >= 0");
+  return rdf_normalize(hist, nbuckets, dim, bucket_width, pairs, volume, g, (cudaStream_t)stream);
+}
+
+int tbs_rdf(const float* points, int64_t n, int dim, float bucket_width, int nbuckets, double volume, double* g) {
+  g_err.clear();
+  if (nbuckets < 1 || nbuckets >= TBS_MAX_BUCKETS) return fail(TBS_EINVAL, "nbuckets out of range");
+  return run_simple(points, n, dim, g, (size_t)nbuckets * 8, [&](tbs_args* a, void* out) {
+    return rdf_impl(a, bucket_width, nbuckets, volume, (double*)out);
+  });
 }
 
 int tbs_pairmatrix_hd_ex(const uint16_t* features, int64_t n, int d, int64_t row_begin, int64_t row_end,
@@ -1062,6 +1213,27 @@ int tbs_peer_free(void* dev_ptr) {
   return TBS_OK;
 }
 
+int tbs_peer_atomics_ok(const char* pci_bus_id, int* ok) {
+  g_err.clear();
+  if (!pci_bus_id || !ok) return fail(TBS_EINVAL, "tbs_peer_atomics_ok: bad arguments");
+  *ok = 0;
+  int self = 0, peer = -1;
+  TBS_CUDA(cudaGetDevice(&self));
+  if (cudaDeviceGetByPCIBusId(&peer, pci_bus_id) != cudaSuccess) {
+    cudaGetLastError();
+    return TBS_OK;   // not visible to this process: no peer access to query
+  }
+  if (peer == self) {
+    *ok = 1;          // the same GPU (e.g. two processes on one device): device-local atomics
+    return TBS_OK;
+  }
+  int access = 0, atomics = 0;
+  TBS_CUDA(cudaDeviceCanAccessPeer(&access, self, peer));
+  TBS_CUDA(cudaDeviceGetP2PAttribute(&atomics, cudaDevP2PAttrNativeAtomicSupported, self, peer));
+  *ok = (access && atomics) ? 1 : 0;
+  return TBS_OK;
+}
+
 const char* tbs_last_error(void) { return g_err.c_str(); }
 
 void tbs_release(void) {
@@ -1076,6 +1248,6 @@ void tbs_release(void) {
 
 uint64_t tbs_launch_count(void) { return g_launches.load(); }
 
-int tbs_version(void) { return 100; }
+int tbs_version(void) { return 200; }
 
 }  // extern "C"

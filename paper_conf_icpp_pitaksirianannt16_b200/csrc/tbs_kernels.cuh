@@ -25,8 +25,16 @@ namespace tbs {
 #ifndef TBS_PUNROLL
 #define TBS_PUNROLL 1                      // partner-quad loop unroll (software-pipelining freedom)
 #endif
+#ifndef TBS_SW_SQRT
+#define TBS_SW_SQRT 0                      // float SDH: (partner q, anchor pair m) slots, bit 4q+m, whose
+#endif                                     // square roots run on the FMA pipe (sqrt_sw2) instead of MUFU
 constexpr int kThreads = 256;              // 8 warps per CTA
 constexpr int kPUnroll = TBS_PUNROLL;
+constexpr unsigned kSwSqrtMask = TBS_SW_SQRT;
+#ifndef TBS_PARTNER_PATH
+#define TBS_PARTNER_PATH 0                 // Fig. 9 ablation (A/B builds only): how partners reach the
+#endif                                     // threads, see run_chunk
+constexpr int kPartnerPath = TBS_PARTNER_PATH;
 constexpr int kWarps = kThreads / 32;
 constexpr int kPadAlign = 4096;            // SoA rows padded to a multiple of every anchor tile / chunk
 constexpr uint32_t kMagic = 0x4B000000u;   // bits of 2^23: x + 2^23 (round-down) = 2^23 + floor(x)
@@ -88,7 +96,9 @@ __device__ __forceinline__ float ord2f(uint32_t o) {
 }
 
 // `pad` is the coordinate value of pad points i >= n (0; +inf for kNN, so pad partners never
-// enter a neighbour list).
+// enter a neighbour list). Coordinates c >= dim of real points (dim 1, 2 padded to D = 3) are 0
+// and enter the bounding box as such. bbox[2D] bit 0: a non-finite coordinate; bit 1: a
+// non-integer coordinate (TBS_VALIDATE under TBS_EXACT_LATTICE).
 __global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_pad, int D, float pad,
                            float* __restrict__ soa, unsigned long long* __restrict__ zero, long long zero_words,
                            uint32_t* __restrict__ bbox) {
@@ -96,19 +106,28 @@ __global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_
   uint32_t lo[4] = {0u, 0u, 0u, 0u}, hi[4] = {0u, 0u, 0u, 0u}, bad = 0u;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n_pad; i += stride) {
     for (int c = 0; c < D; ++c) {
-      float v = i < n ? 0.0f : pad;
-      if (i < n && c < dim) {
-        v = __ldg(pts + i * dim + c);
+      float v = pad;
+      if (i < n) {
+        v = c < dim ? __ldg(pts + i * dim + c) : 0.0f;
         const uint32_t o = f2ord(v);
         lo[c] = max(lo[c], ~o);
         hi[c] = max(hi[c], o);
-        bad |= isfinite(v) ? 0u : 1u;
+        bad |= (isfinite(v) ? 0u : 1u) | (v == rintf(v) ? 0u : 2u);
       }
       soa[(long long)c * n_pad + i] = v;
     }
   }
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < zero_words; i += stride) zero[i] = 0ull;
   if (bbox) {
+    // One-CTA launch (small problems): reduce in shared memory and write the whole 64-byte
+    // block (box, flags, zeroed work-queue counter), so the caller needs no memset before it.
+    __shared__ uint32_t sb[16];
+    const bool one = gridDim.x == 1;
+    if (one) {
+      if (threadIdx.x < 16) sb[threadIdx.x] = 0u;
+      __syncthreads();
+    }
+    uint32_t* dst = one ? sb : bbox;
     for (int c = 0; c < D; ++c) {
       uint32_t a = lo[c], b = hi[c];
 #pragma unroll
@@ -117,18 +136,23 @@ __global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_
         b = max(b, __shfl_xor_sync(0xffffffffu, b, off));
       }
       if ((threadIdx.x & 31) == 0) {
-        if (a) atomicMax(bbox + c, a);
-        if (b) atomicMax(bbox + D + c, b);
+        if (a) atomicMax(dst + c, a);
+        if (b) atomicMax(dst + D + c, b);
       }
     }
-    bad = __any_sync(0xffffffffu, bad != 0u) ? 1u : 0u;
-    if ((threadIdx.x & 31) == 0 && bad) atomicOr(bbox + 2 * D, 1u);
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) bad |= __shfl_xor_sync(0xffffffffu, bad, off);
+    if ((threadIdx.x & 31) == 0 && bad) atomicOr(dst + 2 * D, bad);
+    if (one) {
+      __syncthreads();
+      if (threadIdx.x < 16) bbox[threadIdx.x] = sb[threadIdx.x];
+    }
   }
 }
 
 // Upper bound on any pair distance from the loader's bounding box (+inf if unknown).
 __device__ __forceinline__ float bbox_diameter(const uint32_t* __restrict__ bbox, int D) {
-  if (bbox == nullptr || bbox[2 * D] != 0u) return __int_as_float(0x7f800000);
+  if (bbox == nullptr || (bbox[2 * D] & 1u) != 0u) return __int_as_float(0x7f800000);
   double s = 0.0;
   for (int c = 0; c < D; ++c) {
     if (bbox[c] == 0u || bbox[D + c] == 0u) return __int_as_float(0x7f800000);
@@ -139,11 +163,12 @@ __device__ __forceinline__ float bbox_diameter(const uint32_t* __restrict__ bbox
 }
 
 // ------------------------------------------------------------------------------------
-// Where the Type-I / Type-II flushes land (a9, a12). n == 0: the caller's buffer p[0]
-// (device-scope atomics). n >= 1 (TBS_OUT_PEERS, the fused multi-GPU combine): every
-// rank's buffer p[0..n) — local or mapped from a peer GPU over NVLink by CUDA IPC — gets
-// every flushed partial with a system-scope atomic add, so when all ranks' kernels have
-// completed each buffer holds the all-reduced sum without a separate collective.
+// Where the Type-I / Type-II flushes land (a9, a12). n == 0: the buffer p[0] (device-scope
+// atomics): the caller's output, or under TBS_OUT_PEERS the call's local accumulator. n >= 1
+// (push_peers, the second stage of the fused multi-GPU combine): every rank's buffer p[0..n)
+// — local or mapped from a peer GPU over NVLink by CUDA IPC — gets the partial with a
+// system-scope atomic add, so when all ranks' calls have completed each buffer holds the
+// all-reduced sum without a separate collective.
 // ------------------------------------------------------------------------------------
 constexpr int kMaxPeers = 16;
 struct OutSink {
@@ -292,32 +317,48 @@ struct SdhSmemOp {
     k1 = (uint32_t)min(b1 + (d1.y <= 0.f ? 1 : 0) - (d0.y > 0.f ? 1 : 0), nb - 1);
   }
 
+  // Float mode (or the lattice bias-only variant, estimate scale c instead of 1/w): smem word
+  // addresses of the buckets of two pairs from their square roots q.
+  template <int V>
+  __device__ __forceinline__ void float_addr2(float2 q, uint32_t& ad0, uint32_t& ad1, bool& in0, bool& in1) const {
+    const float c = LATTICE ? scale_b : inv_w;
+    float2 y = __ffma2_rd(q, make_float2(c, c), make_float2(kMagicF, kMagicF));
+    if (!LATTICE && V == 1) {
+      y.x = fminf(y.x, ymax);
+      y.y = fminf(y.y, ymax);
+    }
+    // bits(y) = bits(2^23) + k. Funnel shift (bits << S) | (lo >> (32-S)) with S = log2(4R)
+    // and lo = 4 lane_r << (32-S) gives 4 (k R + lane_r) + (bits(2^23) << S); the
+    // CTA-uniform correction (smem base - (bits(2^23) << S)) is recomputed from the smem
+    // symbol so ptxas fuses shift + add into one ALU LEA.HI with a uniform operand.
+    constexpr int S = LOG2R + 2;
+    const uint32_t lo = (uint32_t)((threadIdx.x & (R - 1)) * 4) << (32 - S);
+    const uint32_t ub = smem_addr(tbs_smem) - ((kMagic + (RANGED ? (uint32_t)klo : 0u)) << S);
+    ad0 = __funnelshift_l(lo, __float_as_uint(y.x), S) + ub;
+    ad1 = __funnelshift_l(lo, __float_as_uint(y.y), S) + ub;
+    if (RANGED) {
+      in0 = __float_as_uint(y.x) - (kMagic + (uint32_t)klo) < (uint32_t)rows;
+      in1 = __float_as_uint(y.y) - (kMagic + (uint32_t)klo) < (uint32_t)rows;
+    }
+  }
+
+  // Float mode, unmasked pairs, square roots on the FMA pipe (the TBS_SW_SQRT slots).
+  static constexpr bool kSwCapable = !LATTICE && !RANGED;
+  template <int V>
+  __device__ __forceinline__ void pair2_sw(float2 s) {
+    uint32_t ad0, ad1;
+    bool in0 = true, in1 = true;
+    float_addr2<V>(sqrt_sw2(s), ad0, ad1, in0, in1);
+    red_smem_inc(ad0);
+    red_smem_inc(ad1);
+  }
+
   template <bool MASKED, int V>
   __device__ __forceinline__ void pair2(float2 s, int pv, int a0, int a1) {
     uint32_t ad0, ad1;
     bool in0 = true, in1 = true;
     if (!LATTICE || V == 4) {
-      // float mode, or the lattice bias-only variant (estimate scale c instead of 1/w)
-      const float c = LATTICE ? scale_b : inv_w;
-      const float2 q = make_float2(sqrt_approx(s.x), sqrt_approx(s.y));
-      float2 y = __ffma2_rd(q, make_float2(c, c), make_float2(kMagicF, kMagicF));
-      if (!LATTICE && V == 1) {
-        y.x = fminf(y.x, ymax);
-        y.y = fminf(y.y, ymax);
-      }
-      // bits(y) = bits(2^23) + k. Funnel shift (bits << S) | (lo >> (32-S)) with S = log2(4R)
-      // and lo = 4 lane_r << (32-S) gives 4 (k R + lane_r) + (bits(2^23) << S); the
-      // CTA-uniform correction (smem base - (bits(2^23) << S)) is recomputed from the smem
-      // symbol so ptxas fuses shift + add into one ALU LEA.HI with a uniform operand.
-      constexpr int S = LOG2R + 2;
-      const uint32_t lo = (uint32_t)((threadIdx.x & (R - 1)) * 4) << (32 - S);
-      const uint32_t ub = smem_addr(tbs_smem) - ((kMagic + (RANGED ? (uint32_t)klo : 0u)) << S);
-      ad0 = __funnelshift_l(lo, __float_as_uint(y.x), S) + ub;
-      ad1 = __funnelshift_l(lo, __float_as_uint(y.y), S) + ub;
-      if (RANGED) {
-        in0 = __float_as_uint(y.x) - (kMagic + (uint32_t)klo) < (uint32_t)rows;
-        in1 = __float_as_uint(y.y) - (kMagic + (uint32_t)klo) < (uint32_t)rows;
-      }
+      float_addr2<V>(make_float2(sqrt_approx(s.x), sqrt_approx(s.y)), ad0, ad1, in0, in1);
     } else if (V == 0) {
       // Lattice, fast variant. The estimate uses a scale rounded UP by 2^-17, far above the
       // sqrt.approx + rounding error (~2^-22) and far below 1/x (x = sqrt(4^j s)/m < 4096),
@@ -356,12 +397,14 @@ struct SdhSmemOp {
       ad0 = (k0 << (LOG2R + 2)) + lb;
       ad1 = (k1 << (LOG2R + 2)) + lb;
     }
-    if (RANGED) {
-      red_smem_inc_if(ad0, in0 && (!MASKED || pv > a0));
-      red_smem_inc_if(ad1, in1 && (!MASKED || pv > a1));
-    } else if (MASKED) {
-      red_smem_inc_gt(ad0, pv, a0);
-      red_smem_inc_gt(ad1, pv, a1);
+    if (RANGED || MASKED) {
+      // Masked pairs (i >= j, pad partners: their distance can leave the histogram) and
+      // out-of-pass buckets add 0 to the lane's own row-0 word: no branch, and the address
+      // stays inside the histogram.
+      const uint32_t safe = smem_addr(tbs_smem) + (uint32_t)((threadIdx.x & (R - 1)) * 4);
+      const bool c0 = in0 && (!MASKED || pv > a0), c1 = in1 && (!MASKED || pv > a1);
+      red_smem_add(c0 ? ad0 : safe, c0 ? 1u : 0u);
+      red_smem_add(c1 ? ad1 : safe, c1 ? 1u : 0u);
     } else {
       red_smem_inc(ad0);
       red_smem_inc(ad1);
@@ -412,6 +455,7 @@ struct SdhGlobalOp {
   int flush_every;           // unused
   const OutSink* out;        // unused (the reduce kernel writes the sink)
 
+  static constexpr bool kSwCapable = false;
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) { mine = part + (size_t)(blockIdx.x % G) * nb; }
   __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
@@ -456,6 +500,7 @@ struct PcfOp {
   const OutSink* out;        // u64 count (or every rank's): the kernel's sink parameter
   uint32_t c;                // per-item counter (<= KA * TP)
   unsigned long long total;  // per-thread running total
+  static constexpr bool kSwCapable = false;
 
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) { c = 0u; total = 0ull; }
@@ -504,6 +549,7 @@ struct KdeOp {
   float2 part;              // current group partial (two lanes of the packed pair)
   float tot, comp;          // Kahan running sum
   const OutSink* out;       // unused
+  static constexpr bool kSwCapable = false;
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) {
     part = make_float2(0.f, 0.f);
@@ -576,13 +622,36 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
     }
   }
   const int n = g.n;
+  // Partner path (the paper's Fig. 9 comparison, L1183-1221; product = 0):
+  //   0  chunk staged in shared memory by TMA bulk copy, read as LDS.128 broadcasts (B = smem);
+  //   1  Alg. 4 register sharing: each lane loads one partner per 32 from global memory (L1)
+  //      and the warp broadcasts it with 3 SHFL per partner (B = global chunk);
+  //   2  read-only L1 path: LDG.128 broadcasts straight from the global SoA (B = global chunk).
+  float sh[D];
 #pragma unroll kPUnroll
   for (int p = 0; p < cnt; p += 4) {
     float c4[D][4];
+    if constexpr (kPartnerPath == 0) {
 #pragma unroll
-    for (int c = 0; c < D; ++c) {
-      const float4 v = *reinterpret_cast<const float4*>(B + c * C::TP + p);
-      c4[c][0] = v.x; c4[c][1] = v.y; c4[c][2] = v.z; c4[c][3] = v.w;
+      for (int c = 0; c < D; ++c) {
+        const float4 v = *reinterpret_cast<const float4*>(B + c * C::TP + p);
+        c4[c][0] = v.x; c4[c][1] = v.y; c4[c][2] = v.z; c4[c][3] = v.w;
+      }
+    } else if constexpr (kPartnerPath == 2) {
+#pragma unroll
+      for (int c = 0; c < D; ++c) {
+        const float4 v = __ldg(reinterpret_cast<const float4*>(B + (long long)c * g.n_pad + p));
+        c4[c][0] = v.x; c4[c][1] = v.y; c4[c][2] = v.z; c4[c][3] = v.w;
+      }
+    } else {
+      if ((p & 31) == 0) {
+#pragma unroll
+        for (int c = 0; c < D; ++c) sh[c] = __ldg(B + (long long)c * g.n_pad + p + (threadIdx.x & 31));
+      }
+#pragma unroll
+      for (int c = 0; c < D; ++c)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) c4[c][q] = __shfl_sync(0xffffffffu, sh[c], (p & 31) + q);
     }
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
@@ -596,6 +665,12 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
         for (int c = 1; c < D; ++c) {
           d = __fadd2_rn(na[c][m], make_float2(c4[c][q], c4[c][q]));
           s = __ffma2_rn(d, d, s);
+        }
+        if constexpr (Op::kSwCapable && !MASKED && kSwSqrtMask != 0u && V <= 1) {
+          if ((kSwSqrtMask >> (q * 4 + m)) & 1u) {   // resolved at compile time (q, m unrolled)
+            op.template pair2_sw<V>(s);
+            continue;
+          }
         }
         op.template pair2<MASKED, V>(s, pv, MASKED ? aidx[2 * m] : 0, MASKED ? aidx[2 * m + 1] : 0);
       }
@@ -645,7 +720,7 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
     if (it < g.items) {
       chunk_end = min(it + g.chunk, g.items);
       item_to_tile(g, it, I, J);
-      issue_chunk<D, C::TP>(soa, g, J, bufs, bar0);
+      if (kPartnerPath == 0) issue_chunk<D, C::TP>(soa, g, J, bufs, bar0);
     }
     s_it[0] = it; s_I[0] = I; s_J[0] = J;
   }
@@ -670,7 +745,7 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
             item_to_tile(g, nit, nI, nJ);
           }
         }
-        if (nit < g.items) issue_chunk<D, C::TP>(soa, g, nJ, bufs + (s ^ 1) * D * C::TP, s ? bar0 : bar1);
+        if (kPartnerPath == 0 && nit < g.items) issue_chunk<D, C::TP>(soa, g, nJ, bufs + (s ^ 1) * D * C::TP, s ? bar0 : bar1);
         s_it[s ^ 1] = nit; s_I[s ^ 1] = nI; s_J[s ^ 1] = nJ;
       }
       if (I != curI) {
@@ -685,9 +760,11 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
           }
         }
       }
-      mbar_wait(s ? bar1 : bar0, (phase >> s) & 1u);
-      phase ^= 1u << s;
-      const float* B = bufs + s * D * C::TP;
+      if (kPartnerPath == 0) {
+        mbar_wait(s ? bar1 : bar0, (phase >> s) & 1u);
+        phase ^= 1u << s;
+      }
+      const float* B = kPartnerPath == 0 ? bufs + s * D * C::TP : soa + (long long)J * C::TP;
       const int p0 = J * C::TP;
       const int cnt = min(C::TP, g.n - p0);
       const bool fast =
@@ -746,6 +823,18 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
     g.trace[3 * blockIdx.x + 1] = t_start;
     g.trace[3 * blockIdx.x + 2] = t_end;
   }
+}
+
+// Fused multi-GPU combine, second stage (TBS_OUT_PEERS): the call's kernels accumulated this
+// rank's partial in a local buffer with device-scope atomics; one thread per word adds it into
+// every rank's output buffer with system-scope atomics (words x ranks remote adds per rank,
+// instead of one add per flushing CTA), then fences them before the kernel completes.
+__global__ void push_peers(const unsigned long long* __restrict__ acc, int words, OutSink out) {
+  for (int k = blockIdx.x * blockDim.x + threadIdx.x; k < words; k += gridDim.x * blockDim.x) {
+    const unsigned long long v = acc[k];
+    if (v) out.add(k, v);
+  }
+  out.fence();
 }
 
 // Sum G partial global copies into the output (one thread per bin, the paper's

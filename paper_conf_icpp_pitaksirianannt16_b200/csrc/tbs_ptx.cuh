@@ -47,21 +47,11 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t
 __device__ __forceinline__ void red_smem_inc(uint32_t addr) {
   asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(addr));
 }
-// Same, predicated on (p > a) — the i<j / tail / row-range mask (one ISETP).
-__device__ __forceinline__ void red_smem_inc_gt(uint32_t addr, int p, int a) {
-  asm volatile(
-      "{\n.reg .pred q;\n"
-      "setp.gt.s32 q, %1, %2;\n"
-      "@q red.shared.add.u32 [%0], 1;\n}\n" ::"r"(addr),
-      "r"(p), "r"(a));
-}
-// Same, predicated on a computed condition (bucket-range passes).
-__device__ __forceinline__ void red_smem_inc_if(uint32_t addr, bool c) {
-  asm volatile(
-      "{\n.reg .pred q;\n"
-      "setp.ne.s32 q, %1, 0;\n"
-      "@q red.shared.add.u32 [%0], 1;\n}\n" ::"r"(addr),
-      "r"((int)c));
+// Add v (0 or 1) to a u32 counter in shared memory (SASS: ATOMS.ADD). The masked pairs of
+// diagonal / ragged / row-range items use this with v = [mask] instead of a predicated
+// increment, which ptxas turns into a branch (BSSY/BRA/BSYNC) around every ATOMS.
+__device__ __forceinline__ void red_smem_add(uint32_t addr, uint32_t v) {
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(addr), "r"(v));
 }
 // Global u64 increment (partially privatised global histogram, SASS: REDG.E.ADD.64).
 // System-scope u64 add (peer memory mapped over NVLink / CUDA IPC: the fused combine).
@@ -86,6 +76,26 @@ __device__ __forceinline__ float sqrt_approx(float x) {
   asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
   return r;
 }
+// Square root of two values on the FMA pipe (no MUFU), for a fraction of the SDH's pairs when
+// the XU pipe is the bound: a magic-constant reciprocal square root with one
+// modified Newton step (constants of Moroz et al., |rel err| <= 6.5e-4), y = s r, then two
+// Newton corrections y += (s - y^2) r / 2. 10 FP32 lane-ops + 2 ALU ops per value; max relative
+// error 2^-24 over [1, 4) and the integers < 2^24 (exhaustive on the GPU: tools/sqrt_bound.cu),
+// i.e. tighter than sqrt.approx. s = 0 gives 0; denormal s gives a value < 1e-19.
+__device__ __forceinline__ float2 sqrt_sw2(float2 s) {
+  float2 r = make_float2(__uint_as_float(0x5F1FFFF9u - (__float_as_uint(s.x) >> 1)),
+                         __uint_as_float(0x5F1FFFF9u - (__float_as_uint(s.y) >> 1)));
+  const float2 t = __fmul2_rn(s, r);
+  const float2 u = __ffma2_rn(make_float2(-t.x, -t.y), r, make_float2(2.38924456f, 2.38924456f));
+  r = __fmul2_rn(__fmul2_rn(r, make_float2(0.703952253f, 0.703952253f)), u);
+  float2 y = __fmul2_rn(s, r);
+  const float2 hr = __fmul2_rn(r, make_float2(0.5f, 0.5f));
+  float2 e = __ffma2_rn(make_float2(-y.x, -y.y), y, s);
+  y = __ffma2_rn(e, hr, y);
+  e = __ffma2_rn(make_float2(-y.x, -y.y), y, s);
+  return __ffma2_rn(e, hr, y);
+}
+
 __device__ __forceinline__ float ex2_approx(float x) {
   float r;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));

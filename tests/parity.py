@@ -3,11 +3,14 @@ import numpy as np
 import oracle
 
 
-def check_sdh_float(h_gpu, h_or, amb):
+def check_sdh_float(h_gpu, h_or, amb, amb_diag=None):
     """Float SDH: mass equal exactly; for every edge e, the cumulative counts
     C(e) = sum_{b<e} h[b] differ by at most A_e (pairs within 1e-6 e w of edge e —
     only those can change side under fp32 rounding). Implies per-bucket
-    |h_gpu[b] - h_or[b]| <= A_b + A_{b+1}. Returns diagnostics."""
+    |h_gpu[b] - h_or[b]| <= A_b + A_{b+1}. Returns diagnostics; with amb_diag (the oracle's
+    5e-7 band counts, oracle.sdh_bands) also the SURVEY §8(c) diagnostic: the edges where the
+    GPU moved more pairs than lie within 5e-7 of the edge, and the excess (a lower bound on
+    the pairs the GPU placed wrongly although they are 5e-7..1e-6 from the edge)."""
     g = np.asarray(h_gpu, dtype=np.int64)
     o = np.asarray(h_or, dtype=np.int64)
     a = np.asarray(amb, dtype=np.int64)
@@ -21,7 +24,15 @@ def check_sdh_float(h_gpu, h_or, amb):
     per = np.abs(g - o)
     lim = a[:nb] + a[1:nb + 1]
     assert np.all(per <= lim)
-    return dict(max_bucket_diff=int(per.max()), edges_differing=int((dev > 0).sum()), amb_total=int(a.sum()))
+    out = dict(max_bucket_diff=int(per.max()), edges_differing=int((dev > 0).sum()), amb_total=int(a.sum()),
+               pairs_moved=int(dev.sum()))
+    if amb_diag is not None:
+        a2 = np.asarray(amb_diag, dtype=np.int64)[1:nb]
+        over = dev - a2
+        out.update(amb_diag_total=int(a2.sum()), edges_over_diag_band=int((over > 0).sum()),
+                   diag_band_excess=int(np.clip(over, 0, None).sum()),
+                   max_dev_over_diag_amb=float(np.max(dev / np.maximum(a2, 1))) if dev.size else 0.0)
+    return out
 
 
 def check_pcf_float(c_gpu, c_or, amb):

@@ -37,7 +37,7 @@ def test_exports_match_header(L):
 
 
 def test_version(L):
-    assert tbs.version() == 100
+    assert tbs.version() == 200
 
 
 def test_kernels_are_sm100a(L):
@@ -50,7 +50,7 @@ def test_kernels_are_sm100a(L):
 
 
 def _args(n=10, dim=3, rb=0, re_=None, pts=1):
-    return tbs._Args(pts, n, dim, rb, n if re_ is None else re_, None, 0, None, None)
+    return tbs._Args(pts, n, dim, rb, n if re_ is None else re_, None, 0, None, None, None, 0, 0)
 
 
 @pytest.mark.parametrize("kw,nb,w", [
@@ -72,6 +72,25 @@ def test_sdh_einval_null_hist_and_lattice_width(L):
     h = np.zeros(8, np.uint64)
     assert L.tbs_sdh_ex(ctypes.byref(a), 0.3, 8, h.ctypes.data) == tbs.TBS_EINVAL      # 0.3 is not m * 2^-j
     assert "EXACT_LATTICE" in tbs.last_error()
+
+
+def test_rdf_einval(L):
+    """RDF (NEXT-1): argument errors are synchronous (no GPU work)."""
+    a = _args()
+    g = np.zeros(8, np.float64)
+    assert L.tbs_rdf_ex(ctypes.byref(a), 0.5, 8, 0.0, g.ctypes.data) == tbs.TBS_EINVAL           # volume
+    assert L.tbs_rdf_ex(ctypes.byref(a), 0.5, 8, float("inf"), g.ctypes.data) == tbs.TBS_EINVAL
+    assert L.tbs_rdf_ex(ctypes.byref(a), 0.5, 0, 1.0, g.ctypes.data) == tbs.TBS_EINVAL
+    assert L.tbs_rdf_ex(ctypes.byref(a), -0.5, 8, 1.0, g.ctypes.data) == tbs.TBS_EINVAL
+    assert L.tbs_rdf_ex(ctypes.byref(a), 0.5, 8, 1.0, None) == tbs.TBS_EINVAL
+    a.flags = tbs.TBS_OUT_PEERS
+    assert L.tbs_rdf_ex(ctypes.byref(a), 0.5, 8, 1.0, g.ctypes.data) == tbs.TBS_EUNSUPPORTED
+    h = np.zeros(8, np.uint64)
+    assert L.tbs_rdf_hist_ex(h.ctypes.data, 8, 5, 0.5, 10.0, 1.0, g.ctypes.data, None) == tbs.TBS_EINVAL  # dim
+    assert L.tbs_rdf_hist_ex(h.ctypes.data, 8, 3, 0.5, -1.0, 1.0, g.ctypes.data, None) == tbs.TBS_EINVAL  # pairs
+    assert L.tbs_rdf_hist_ex(None, 8, 3, 0.5, 10.0, 1.0, g.ctypes.data, None) == tbs.TBS_EINVAL
+    ok = ctypes.c_int(7)
+    assert L.tbs_peer_atomics_ok(None, ctypes.byref(ok)) == tbs.TBS_EINVAL
 
 
 def test_pcf_and_matrix_einval(L):
@@ -99,6 +118,12 @@ def test_out_peers_validation(L):
     assert L.tbs_sdh_ex(ctypes.byref(a), 0.5, 8, None) == tbs.TBS_EINVAL       # a NULL peer
     assert "out_peers[1]" in tbs.last_error()
     arr[1] = 2
+    # every peer buffer must hold exactly the words the call writes
+    a.out_peer_words = 4
+    assert L.tbs_sdh_ex(ctypes.byref(a), 0.5, 8, None) == tbs.TBS_EINVAL       # 4 words < nb = 8
+    assert "out_peer_words" in tbs.last_error()
+    assert L.tbs_pcf_ex(ctypes.byref(a), 0.5, None) == tbs.TBS_EINVAL          # 4 words != 1
+    a.out_peer_words = 8
     c = np.zeros(1, np.float64)
     assert L.tbs_kde_ex(ctypes.byref(a), 1.0, c.ctypes.data) == tbs.TBS_EUNSUPPORTED
     assert L.tbs_pairmatrix_ex(ctypes.byref(a), tbs._Kernel(0, 1.0), c.ctypes.data) == tbs.TBS_EUNSUPPORTED

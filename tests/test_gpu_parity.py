@@ -48,6 +48,27 @@ def test_sdh_uniform_ragged(tbs, n):
     check_sdh_float(h, ho, amb)
 
 
+@pytest.mark.parametrize("kind,nb,offset", [("uniform", 64, 0.0), ("uniform", 256, 0.0), ("uniform", 16384, 0.0),
+                                             ("clustered", 256, 0.0), ("uniform", 256, 1000.0)])
+def test_sdh_diag_band(tbs, kind, nb, offset):
+    """SURVEY §8(c) diagnostic beside the 1e-6 acceptance rule: with the oracle's 5e-7 band
+    counts, no edge may see more pairs moved than lie within 5e-7 of it (the fp32 error budget,
+    DESIGN §10, is <= ~4e-7 relative, whatever the coordinates' offset). The numbers are also
+    appended to gpurun_out/diag_band.jsonl when that directory exists."""
+    import json
+    import os
+    n = 30000
+    p = g.make(kind, n, 90 + nb) + np.float32(offset)
+    w = w_of(nb)
+    h = sdh_gpu(tbs, p, w, nb)
+    ho, amb, amb2 = oracle.sdh_bands(p, w, nb)
+    d = check_sdh_float(h, ho, amb, amb2)
+    if os.path.isdir("gpurun_out"):
+        with open(os.path.join("gpurun_out", "diag_band.jsonl"), "a") as f:
+            f.write(json.dumps(dict(kind=kind, n=n, nb=nb, offset=offset, **d)) + "\n")
+    assert d["edges_over_diag_band"] == 0, d
+
+
 @pytest.mark.parametrize("n", [20001, 30000])
 def test_sdh_main_config_ragged(tbs, n):
     """Sizes above the small-problem switch: the main tile configuration, ragged tail."""
@@ -157,6 +178,8 @@ def test_sqrt_approx_bound():
                     os.path.join(root, "tools", "sqrt_bound.cu")], check=True)
     r = json.loads(subprocess.run([exe], check=True, capture_output=True, text=True).stdout)
     assert r["log2_int"] <= -22.0 and r["log2_1_4"] <= -22.0, r
+    # the FMA-pipe square root (sqrt_sw2, TBS_SW_SQRT slots) is at least as tight as MUFU
+    assert r["sw_log2_int"] <= -23.0 and r["sw_log2_1_4"] <= -23.0, r
 
 
 @pytest.mark.parametrize("mode", [None, "lane", "cta", "global"])
@@ -307,13 +330,61 @@ def test_kde_host_entry_point(tbs):
     assert abs(out[0] - oracle.kde(p, 1.5)) <= 1e-5 * out[0]
 
 
-def test_rdf(tbs):
-    p = g.uniform(20000, 3)
-    w, nb = float(np.float32(math.sqrt(3) / 128)), 128
-    h = sdh_gpu(tbs, p, w, nb)
-    gr = tbs.rdf(dev(p), w, nb, 1.0)
-    np.testing.assert_allclose(gr, oracle.rdf(h, w, 20000, 1.0), rtol=1e-13, atol=0)
-    assert 0.9 < gr[4] < 1.0        # near-ideal at small r, boundary deficit below 1
+def _ideal(w, nb, dim, pairs, volume):
+    """Ideal-gas shell counts with the ball volume from scipy's Gamma function (test side)."""
+    from scipy.special import gamma as G
+    c = math.pi ** (dim / 2) / G(dim / 2 + 1)
+    k = np.arange(nb, dtype=np.float64)
+    return pairs * c * (((k + 1) * w) ** dim - (k * w) ** dim) / volume
+
+
+@pytest.mark.parametrize("dim", [1, 2, 3, 4])
+def test_rdf_lattice_exact_dims(tbs, dim):
+    """RDF (NEXT-1, reading R6) on integer-valued points: the histograms are exact on both
+    sides, so g agrees to the rounding of two independently written normalisations."""
+    import torch
+    n, nb, w = 6000, 48, 0.5
+    p = np.floor(g.uniform(n, 60 + dim, dim) * 40.0).astype(np.float32)
+    gr = tbs.rdf(dev(p), w, nb, 40.0 ** dim, lattice=True)
+    torch.cuda.synchronize()
+    go, ho, _ = oracle.rdf_points(p, w, nb, 40.0 ** dim, lattice=(1, 1))
+    assert ho[:nb].sum() > 0
+    np.testing.assert_allclose(gr.cpu().numpy(), go, rtol=1e-12, atol=0)
+
+
+@pytest.mark.parametrize("dim,rows", [(1, None), (2, None), (3, None), (4, None), (3, (1000, 7777))])
+def test_rdf_float_dims(tbs, dim, rows):
+    """Float inputs: the GPU's g may differ from the oracle's only through pairs within the
+    1e-6 band of an edge, so |g_gpu[k] - g_or[k]| <= (A_k + A_{k+1}) / ideal_k (A from the
+    ORACLE's band counts, ideal_k from the test's own ball volume) + rounding; the whole
+    vector is also within that bound of the oracle pipeline on a row strip."""
+    import torch
+    n, nb = 9000, 64
+    w = float(np.float32(math.sqrt(dim) / nb))
+    p = g.uniform(n, 70 + dim, dim)
+    gr = tbs.rdf(dev(p), w, nb, 1.0, rows=rows).cpu().numpy()
+    torch.cuda.synchronize()
+    go, ho, amb = oracle.rdf_points(p, w, nb, 1.0, rows=rows)
+    ideal = _ideal(np.float64(np.float32(w)), nb, dim, oracle.pairs_of_rows(n, rows), 1.0)
+    a = amb.astype(np.float64)
+    bound = (a[:nb] + a[1:nb + 1]) / ideal + 1e-12 * np.abs(go)
+    assert np.all(np.abs(gr - go) <= bound), np.max(np.abs(gr - go) - bound)
+    np.testing.assert_allclose(go, ho[:nb] / ideal, rtol=1e-9)   # the test's ideal = the oracle's
+
+
+def test_rdf_host_entry_and_degenerate(tbs):
+    """tbs_rdf with host buffers equals the device path; n < 2 gives g = 0; a pair beyond
+    nb w (clamp bucket) never enters g."""
+    import ctypes
+    p = g.uniform(3000, 77)
+    nb, w = 32, 0.05
+    out = np.zeros(nb, np.float64)
+    assert tbs.lib().tbs_rdf(p.ctypes.data, 3000, 3, ctypes.c_float(w), nb, ctypes.c_double(1.0),
+                             out.ctypes.data) == 0, tbs.last_error()
+    np.testing.assert_array_equal(out, tbs.rdf(dev(p), w, nb, 1.0).cpu().numpy())
+    assert not tbs.rdf(dev(p[:1]), w, nb, 1.0).cpu().numpy().any()
+    q = np.array([[0, 0, 0], [5, 0, 0]], np.float32)
+    assert not tbs.rdf(dev(q), w, nb, 1.0).cpu().numpy().any()
 
 
 # ------------------------------------------------------------------ output-stage replication R and bucket-range passes
@@ -518,3 +589,36 @@ def test_knn_host_entry_point_and_einval(tbs):
         tbs.knn(dev(p), 33)
     with pytest.raises(tbs.TbsError):
         tbs.knn(dev(p), 0)
+
+
+# ------------------------------------------------------------------ TBS_VALIDATE (SURVEY §8(b) debug flag)
+def test_validate_flag(tbs):
+    """The debug flag checks what the loader recorded before any pair kernel runs: non-finite
+    coordinates (SDH, 2PCF, RDF) and, under TBS_EXACT_LATTICE, non-integer coordinates or a
+    bounding box whose squared pair distances could reach 2^24. Valid inputs give the same
+    result as without the flag."""
+    import torch
+    lat = g.lattice(12, 3)
+    ok = tbs.sdh(dev(lat), 0.5, 40, lattice=True, validate=True)
+    assert ok.cpu().tolist() == tbs.sdh(dev(lat), 0.5, 40, lattice=True).cpu().tolist()
+    bad = lat.copy()
+    bad[7, 1] = 3.5                                   # not integer-valued
+    with pytest.raises(tbs.TbsError, match="integer-valued"):
+        tbs.sdh(dev(bad), 0.5, 40, lattice=True, validate=True)
+    wide = lat.copy()
+    wide[0] = (0, 0, 0)
+    wide[1] = (5000, 0, 0)                            # 5000^2 >= 2^24
+    with pytest.raises(tbs.TbsError, match="2\\^24"):
+        tbs.sdh(dev(wide), 1.0, 40, lattice=True, validate=True)
+    p = g.uniform(3000, 5)
+    p[100, 2] = np.nan
+    for call in (lambda x: tbs.sdh(x, 0.01, 64, validate=True), lambda x: tbs.pcf(x, 0.1, validate=True),
+                 lambda x: tbs.rdf(x, 0.01, 64, 1.0, validate=True)):
+        with pytest.raises(tbs.TbsError, match="non-finite"):
+            call(dev(p))
+    p[100, 2] = np.inf
+    with pytest.raises(tbs.TbsError, match="non-finite"):
+        tbs.sdh(dev(p), 0.01, 64, validate=True)
+    q = g.uniform(3000, 5)                            # float data passes (non-integer is fine)
+    assert int(tbs.sdh(dev(q), 0.01, 64, validate=True).sum().item()) == 3000 * 2999 // 2
+    torch.cuda.synchronize()

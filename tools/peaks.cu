@@ -140,6 +140,32 @@ __global__ void k_atoms_pure(unsigned* out) {
   if (threadIdx.x == 0 && h[5] == 0xffffffffu) out[0] = h[0];
 }
 
+// Random bins over a LARGE histogram (16384 bins), R replicas per bin laid out
+// word[k * R + (lane & (R-1))] exactly as SdhSmemOp<LOG2R>: the bank of a lane's increment is
+// random, so a warp's ATOMS costs max-bank-load wavefronts. Occupancy set by the launch.
+template <int LOG2R>
+__global__ void k_atoms_big(unsigned* out, int log2bins) {
+  extern __shared__ unsigned h[];
+  const int lane = threadIdx.x & 31;
+  const int words = (1 << log2bins) << LOG2R;
+  for (int i = threadIdx.x; i < words; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  unsigned k[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) k[c] = (threadIdx.x * 2654435761u + blockIdx.x * 97u) ^ (c * 40503u);
+  const uint32_t base = (uint32_t)__cvta_generic_to_shared(h) + (uint32_t)((lane & ((1 << LOG2R) - 1)) * 4);
+  const int sh = 32 - log2bins;
+  for (int i = 0; i < ITERS / 4; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      k[c] = k[c] * 1664525u + 1013904223u;
+      asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(base + ((k[c] >> sh) << (LOG2R + 2))));
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0 && h[5] == 0xffffffffu) out[0] = h[0];
+}
+
 // ---- LDS.128 broadcast ---------------------------------------------------------
 __global__ void k_lds128(float* out) {
   __shared__ float4 s[1024];
@@ -195,6 +221,22 @@ int main() {
   rep("atoms_pure_lane_private", at, timeit([&] { k_atoms_pure<<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
   rep("atoms_random_256", at, timeit([&] { k_atoms<1><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
   rep("atoms_same_addr", at, timeit([&] { k_atoms<2><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  // C4's access pattern: 16384 random bins, R = 2 replicas (128 KB: one 256-thread CTA per SM),
+  // R = 1 (64 KB: 1, 2 or 3 CTAs per SM), and 512-thread CTAs sharing the R = 2 copies
+  CK(cudaFuncSetAttribute(k_atoms_big<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 16384 * 2 * 4));
+  CK(cudaFuncSetAttribute(k_atoms_big<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 16384 * 4));
+  auto atoms_big = [&](const char* name, int log2r, int cta_per_sm, int thr_per_cta) {
+    const double ops = (double)(ITERS / 4) * 8 * sms * cta_per_sm * thr_per_cta;
+    const size_t sm_b = (size_t)16384 * 4 << log2r;
+    if (log2r == 1) rep(name, ops, timeit([&] { k_atoms_big<1><<<sms * cta_per_sm, thr_per_cta, sm_b>>>((unsigned*)dout, 14); }));
+    else rep(name, ops, timeit([&] { k_atoms_big<0><<<sms * cta_per_sm, thr_per_cta, sm_b>>>((unsigned*)dout, 14); }));
+  };
+  atoms_big("atoms_random_16k_r2_1x256", 1, 1, 256);
+  atoms_big("atoms_random_16k_r2_1x512", 1, 1, 512);
+  atoms_big("atoms_random_16k_r2_1x1024", 1, 1, 1024);
+  atoms_big("atoms_random_16k_r1_1x256", 0, 1, 256);
+  atoms_big("atoms_random_16k_r1_2x256", 0, 2, 256);
+  atoms_big("atoms_random_16k_r1_3x256", 0, 3, 256);
   rep("lds128_bcast_instr", (double)ITERS * thr, timeit([&] { k_lds128<<<blocks, threads>>>(dout); }));
   size_t bytes = (size_t)8 << 30; float4* big; CK(cudaMalloc(&big, bytes));
   double tw = timeit([&] { k_write<<<sms * 4, 512>>>(big, bytes / 16); });
