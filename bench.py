@@ -299,6 +299,8 @@ def main():
     ap.add_argument("--combine", default="nccl", choices=["nccl", "fused"],
                     help="N > 1, SDH / 2PCF: NCCL all_reduce (default) or the fused peer-memory flush")
     ap.add_argument("--dry-run", action="store_true", help="launch path only (gloo, no GPU work)")
+    ap.add_argument("--graph", default="auto", choices=["auto", "on", "off"],
+                    help="replay each step from a CUDA graph (auto: one GPU, n <= 64K, Type-I/II)")
     args = ap.parse_args()
     if "WORLD_SIZE" not in os.environ and args.gpus > 1:
         return relaunch(args)
@@ -392,6 +394,29 @@ def main():
         flush.fill_(1)
         step()
     torch.cuda.synchronize(dev)
+    # Launch-bound steps (small n, one GPU): capture one step (loader + pair kernel + flush) in a
+    # CUDA graph and replay it, so the timed steps measure the device work, not the host's
+    # per-launch latency. The kernels' own events are not captured: the step events time it.
+    graph, graph_launches = None, 0
+    if args.graph == "on" or (args.graph == "auto" and world == 1 and n <= 65536
+                              and op in ("sdh", "sdh_lattice", "pcf", "kde")):
+        try:
+            side = torch.cuda.Stream(dev)
+            side.wait_stream(st)
+            with torch.cuda.stream(side):
+                step()
+            st.wait_stream(side)
+            torch.cuda.synchronize(dev)
+            graph = torch.cuda.CUDAGraph()
+            lc = tbs.launch_count()
+            with torch.cuda.graph(graph):
+                step()
+            graph_launches = tbs.launch_count() - lc
+            graph.replay()
+            torch.cuda.synchronize(dev)
+        except Exception as e:   # noqa: BLE001 — report and time the plain launches
+            print(f"[bench] CUDA graph capture failed ({e}); timing plain launches", file=sys.stderr)
+            graph = None
     if pg is not None:
         dist.barrier()
     torch.cuda.synchronize(dev)
@@ -405,7 +430,10 @@ def main():
     for k in range(args.steps):
         flush.fill_(k & 0xFF)    # L2 flush between steps (256 MiB > 126 MB L2), outside the step events
         sev[k][0].record(st)
-        step(events=kev[k])
+        if graph is not None:
+            graph.replay()
+        else:
+            step(events=kev[k])
         sev[k][1].record(st)
     t1.record(st)
     torch.cuda.synchronize(dev)
@@ -413,11 +441,12 @@ def main():
         clocks.mark(False)
     if pg is not None:
         dist.barrier()
-    launches = tbs.launch_count() - l0
+    launches = tbs.launch_count() - l0 if graph is None else graph_launches * args.steps
     ck = clocks.stop() if clocks else None
     region_ms = t0.elapsed_time(t1)                          # whole bracket, L2 flushes included
     ms = sum(a.elapsed_time(b) for a, b in sev)               # the K steps themselves
-    kms = [a.elapsed_time(b) for a, b in kev]
+    # the dominant kernel's time: its own events, or under a graph the whole step (conservative)
+    kms = [a.elapsed_time(b) for a, b in (kev if graph is None else sev)]
     if pg is not None:
         tt = torch.tensor([ms, sum(kms) / len(kms), region_ms], dtype=torch.float64, device=dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -440,6 +469,13 @@ def main():
                 "frac": achieved / pk["hbm"], "peak_source": pk["hbm_src"] + " (a read+write copy; this kernel only writes)",
                 "frac_of_nominal": achieved / 7.7e12,   # HGX HBM3e 7.7 TB/s (B200_PROFILING.md), context
                 "algorithmic_bytes_per_launch": bytes_}
+        rp = os.path.join(ROOT, "profiles", "r02_peaks.json")
+        if os.path.exists(rp):
+            # this kernel only WRITES: the measured write-only ceiling (cudaMemset of 8 GiB,
+            # tools/peaks.cu) is the tighter reference than the read+write copy bandwidth
+            wpk = json.load(open(rp))["hbm_memset_GBps"] * 1e9
+            roof["write_peak_GBps"] = wpk / 1e9
+            roof["frac_of_write_peak"] = achieved / wpk
         if op == "pairmatrix_hd":
             # the Gram contraction: 2 d flops per entry on the bf16 tensor cores; the bound is
             # whichever of (output bytes / HBM, flops / tensor peak) takes longer
@@ -482,12 +518,16 @@ def main():
             roof["frac_of_mufu_cap"] = pairs_s / pk["mufu"]
             if nb + 32 > 768:
                 # fewer than 32 lane-private replicas fit (DESIGN.md §7 a8): the increments hit
-                # random banks of one shared copy; the measured ceiling of that access pattern
-                # (tools/peaks.cu, profiles/r01_peaks.json atoms_random_256) bounds this design
-                rp = os.path.join(ROOT, "profiles", "r01_peaks.json")
+                # random banks of R shared copies; the measured ceiling of that access pattern
+                # (tools/peaks.cu, profiles/r02_peaks.json) bounds this design: nb >= 8192 runs
+                # R <= 2 copies in one 256-thread CTA per SM (atoms_random_16k_r2_1x256, C4's exact
+                # layout), smaller nb more replicas (atoms_random_256, one copy: a lower bound)
+                rp = os.path.join(ROOT, "profiles", "r02_peaks.json")
                 if os.path.exists(rp):
-                    cap = json.load(open(rp))["atoms_random_256"]["per_clk_per_sm"] * SMS * pk["f_max"]
+                    key = "atoms_random_16k_r2_1x256" if nb >= 8192 else "atoms_random_256"
+                    cap = json.load(open(rp))[key]["per_clk_per_sm"] * SMS * pk["f_max"]
                     roof["atoms_random_cap"] = cap / 1e9
+                    roof["atoms_random_cap_source"] = f"profiles/r02_peaks.json {key}"
                     roof["frac_of_atoms_random_cap"] = pairs_s / cap
     roof["traffic"] = None
     prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -560,7 +600,7 @@ def main():
                "timed_region_ms": region_ms,
                "parallelism": f"rows{world}" if world > 1 else "single",
                "step": "loader + pair kernel + flush" + (f" + combine ({combine})" if world > 1 else ""),
-               "combine": combine}
+               "combine": combine, "cuda_graph": graph is not None}
         if op == "sdh":
             cfg["bucket_width"] = w
         line = {"metric": METRIC if op in ("sdh", "sdh_lattice") else f"{op} throughput ({unit})",

@@ -76,7 +76,7 @@ using LatFastCfg = Cfg<TBS_LATF_CFG>;
 // Small problems (fewer work items than ~2 per SM with the main configs): finer tiles so
 // the grid covers the GPU (BASELINE configs[0], N = 4096, is launch/latency-bound).
 #ifndef TBS_SMALL_TP
-#define TBS_SMALL_TP 64
+#define TBS_SMALL_TP 128
 #endif
 using SmallCfg = Cfg<2, TBS_SMALL_TP, 4>;
 // Use the small-problem config when the main config yields fewer than this many items per SM.
@@ -189,6 +189,7 @@ int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op
   long long grid = (long long)dev.sms * occ;
   if (grid > g.items) grid = g.items;
   g.chunk = std::max<long long>(1, g.items / (grid * 200));   // ~200 grabs per CTA
+  if (grid == g.items) g.chunk = 0;   // one item per CTA: static assignment, no queue round trips
   static const bool trace_on = getenv("TBS_TRACE") != nullptr;  // debug: CTA residency trace to stderr
   if (trace_on) TBS_CUDA(cudaMalloc(&g.trace, (size_t)grid * 3 * 8));
   if (eb) TBS_CUDA(cudaEventRecord(eb, st));
@@ -476,7 +477,7 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   const long long one_copy_budget = dev.smem_optin - 2ll * 4 * SdhCfg::TP * 4 - 256;
   // Measured on B200 (tools/ab_r.sh, N=1M): the most replicas that fit win even at one CTA
   // per SM, except that R = 32 is only worth it while it leaves room for 2+ CTAs.
-  const long long rows = nb + kGuard;
+  const long long rows = nb + kGuard + 1;   // + the trash row of masked pairs
   if (rows * 32 * 4 <= part_budget) pl.log2r = 5;
   else if (rows * 16 * 4 <= one_copy_budget) pl.log2r = 4;
   else if (rows * 8 * 4 <= one_copy_budget) pl.log2r = 3;
@@ -486,7 +487,7 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   else {
     // beyond one copy: up to 8 bucket-range passes with one copy (each pass ~2.5e12 pairs/s
     // vs ~0.2e12 for L2 atomics), else the partially privatised global histogram
-    const int per_pass = (int)(one_copy_budget / 4) - kGuard;
+    const int per_pass = (int)(one_copy_budget / 4) - kGuard - 1;
     const int passes = (nb + per_pass - 1) / per_pass;
     if (passes <= 8) {
       pl.log2r = 0;
@@ -497,14 +498,14 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
     }
   }
   static const int r_env = [] { const char* e = getenv("TBS_LOG2R"); return e ? atoi(e) : -1; }();  // experiments
-  if (r_env >= 0 && !pl.global && pl.passes == 1 && (long long)(nb + kGuard) * (4ll << r_env) <= one_copy_budget)
+  if (r_env >= 0 && !pl.global && pl.passes == 1 && rows * (4ll << r_env) <= one_copy_budget)
     pl.log2r = r_env;
   if (a->flags & TBS_HIST_FORCE_LANE) {
-    if ((long long)(nb + kGuard) * 32 * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_LANE: nb too large for smem");
+    if (rows * 32 * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_LANE: nb too large for smem");
     pl = SdhPlan{lattice, false, 5};
   }
   if (a->flags & TBS_HIST_FORCE_CTA) {
-    if ((long long)(nb + kGuard) * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_CTA: nb too large for smem");
+    if (rows * 4 > one_copy_budget) return fail(TBS_EUNSUPPORTED, "FORCE_CTA: nb too large for smem");
     pl = SdhPlan{lattice, false, 0};
   }
   if (a->flags & TBS_HIST_FORCE_PASSES) {   // bucket-range passes even when one copy fits (tests)

@@ -189,6 +189,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   }
   hd::tc_fence_before();
   cluster_sync();   // barriers of both CTAs initialised, TMEM allocated, before any remote signal
+  // The CTA barrier repeats what the cluster barrier already ordered (the holder written by
+  // tcgen05.alloc before any thread reads it) in the form compute-sanitizer's racecheck
+  // tracks: it does not model barrier.cluster and reported the holder read as a race (r01).
+  __syncthreads();
   hd::tc_fence_after();
   const uint32_t tmem = *tmem_holder;
 

@@ -62,7 +62,7 @@ struct Geom {
   long long items;  // total work items
   unsigned long long* trace;  // debug only (TBS_TRACE): per CTA {smid, t_start, t_end}, else nullptr
   unsigned long long* counter;  // work-queue head (zeroed by the loader's memset), in items
-  long long chunk;              // items grabbed per atomic
+  long long chunk;              // items grabbed per atomic (0: static, one item per CTA)
 };
 
 __device__ __forceinline__ long long items_before(const Geom& g, long long I) {
@@ -231,7 +231,8 @@ struct SdhSmemOp {
   float ymax;         // float: 2^23 + nb - 1 (clamp variant)
   int flush_every;    // items between overflow flushes
 
-  __host__ __device__ long long smem_bytes() const { return (long long)rows * R * 4; }
+  // rows + 1: the last row is the trash row masked pairs increment (never flushed)
+  __host__ __device__ long long smem_bytes() const { return (long long)(rows + 1) * R * 4; }
 
   __device__ __forceinline__ void init(unsigned char* smem) {
     uint32_t* h = reinterpret_cast<uint32_t*>(smem);
@@ -399,12 +400,13 @@ struct SdhSmemOp {
     }
     if (RANGED || MASKED) {
       // Masked pairs (i >= j, pad partners: their distance can leave the histogram) and
-      // out-of-pass buckets add 0 to the lane's own row-0 word: no branch, and the address
-      // stays inside the histogram.
-      const uint32_t safe = smem_addr(tbs_smem) + (uint32_t)((threadIdx.x & (R - 1)) * 4);
+      // out-of-pass buckets increment the lane's word of the trash row `rows` instead: no
+      // branch (a predicated ATOMS becomes BSSY/BRA/BSYNC), the same ATOMS.POPC.INC, and the
+      // address stays inside the allocation.
+      const uint32_t trash = smem_addr(tbs_smem) + (uint32_t)(((rows << LOG2R) + (threadIdx.x & (R - 1))) * 4);
       const bool c0 = in0 && (!MASKED || pv > a0), c1 = in1 && (!MASKED || pv > a1);
-      red_smem_add(c0 ? ad0 : safe, c0 ? 1u : 0u);
-      red_smem_add(c1 ? ad1 : safe, c1 ? 1u : 0u);
+      red_smem_inc(c0 ? ad0 : trash);
+      red_smem_inc(c1 ? ad1 : trash);
     } else {
       red_smem_inc(ad0);
       red_smem_inc(ad1);
@@ -715,10 +717,11 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
   __shared__ int s_I[2], s_J[2];
   long long it, chunk_end = 0;
   int I = 0, J = 0;
+  // g.chunk == 0: one item per CTA (grid == items, small problems): item = blockIdx.x, no queue
   if (tid == 0) {
-    it = (long long)atomicAdd(g.counter, (unsigned long long)g.chunk);
+    it = g.chunk > 0 ? (long long)atomicAdd(g.counter, (unsigned long long)g.chunk) : (long long)blockIdx.x;
     if (it < g.items) {
-      chunk_end = min(it + g.chunk, g.items);
+      chunk_end = g.chunk > 0 ? min(it + g.chunk, g.items) : it + 1;
       item_to_tile(g, it, I, J);
       if (kPartnerPath == 0) issue_chunk<D, C::TP>(soa, g, J, bufs, bar0);
     }
@@ -739,7 +742,7 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
         if (nit < chunk_end) {
           if (nJ == g.Mc) { nI = I + 1; nJ = nI * C::RATIO; }
         } else {
-          nit = (long long)atomicAdd(g.counter, (unsigned long long)g.chunk);
+          nit = g.chunk > 0 ? (long long)atomicAdd(g.counter, (unsigned long long)g.chunk) : g.items;
           if (nit < g.items) {
             chunk_end = min(nit + g.chunk, g.items);
             item_to_tile(g, nit, nI, nJ);

@@ -47,12 +47,6 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t
 __device__ __forceinline__ void red_smem_inc(uint32_t addr) {
   asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(addr));
 }
-// Add v (0 or 1) to a u32 counter in shared memory (SASS: ATOMS.ADD). The masked pairs of
-// diagonal / ragged / row-range items use this with v = [mask] instead of a predicated
-// increment, which ptxas turns into a branch (BSSY/BRA/BSYNC) around every ATOMS.
-__device__ __forceinline__ void red_smem_add(uint32_t addr, uint32_t v) {
-  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(addr), "r"(v));
-}
 // Global u64 increment (partially privatised global histogram, SASS: REDG.E.ADD.64).
 // System-scope u64 add (peer memory mapped over NVLink / CUDA IPC: the fused combine).
 __device__ __forceinline__ void red_sys_add_u64(unsigned long long* addr, unsigned long long v) {

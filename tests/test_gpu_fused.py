@@ -1,6 +1,6 @@
-"""GPU tests of the fused multi-GPU combine (TBS_OUT_PEERS): the
-SDH / 2PCF flush adds every partial into every rank's buffer (system-scope atomics over
-peer memory) instead of a separate all_reduce.
+"""GPU tests of the fused multi-GPU combine (TBS_OUT_PEERS): each
+SDH / 2PCF call accumulates its strip's partial locally and its last kernel adds it into every
+rank's buffer (system-scope atomics over peer memory) instead of a separate all_reduce.
 
 Only one GPU is available here, so the peers are (1) several local buffers in one process
 (the fan-out itself), and (2) two processes on the same GPU whose buffers are mapped into
@@ -31,7 +31,7 @@ def _fanout(tbs, p, op, npeers, world, **kw):
     flags = tbs.TBS_OUT_PEERS | (tbs.TBS_EXACT_LATTICE if kw.get("lattice") else 0) | tbs.HIST_MODES[kw.get("mode")]
     for r in range(world):
         a, _ = tbs._args(pt, tbs.rank_rows(len(p), world, r), flags, None, None)
-        a.out_peers, a.n_out_peers = arr, npeers
+        a.out_peers, a.n_out_peers, a.out_peer_words = arr, npeers, words
         if op == "sdh":
             rc = tbs.lib().tbs_sdh_ex(ctypes.byref(a), float(kw["w"]), int(kw["nb"]), None)
         else:

@@ -60,9 +60,13 @@ __global__ void intra(const float* __restrict__ pts, int B, float inv_w, unsigne
         if (j > t) inc(h, s, inv_w, lane);
       }
     } else {
-      for (int j = 1; j <= B / 2; ++j) {
-        if (j == B / 2 && t >= B / 2) break;
+      for (int j = 1; j < B / 2; ++j) {
         const int q = (t + j) & (B - 1);
+        const float dx = sx[q] - ax, dy = sy[q] - ay, dz = sz[q] - az;
+        inc(h, fmaf(dz, dz, fmaf(dy, dy, dx * dx)), inv_w, lane);
+      }
+      if (t < B / 2) {                       // the last step: only the lower half (L1094-1097)
+        const int q = t + B / 2;
         const float dx = sx[q] - ax, dy = sy[q] - ay, dz = sz[q] - az;
         inc(h, fmaf(dz, dz, fmaf(dy, dy, dx * dx)), inv_w, lane);
       }

@@ -51,6 +51,44 @@ __global__ void k_ffma2(float* out, float y0, float z0) {
   if (s == 1.2345f) out[0] = s;
 }
 
+// ---- packed FFMA2 and scalar FFMA interleaved on independent chains: does the scalar
+// stream use capacity (fmalite) the packed one leaves idle? Lane-ops = 2 x FFMA2 + FFMA.
+__global__ void k_mix(float* out, float y0, float z0) {
+  float2 y = make_float2(y0 + threadIdx.x * 1e-9f, y0), z = make_float2(z0, z0 - threadIdx.x * 1e-9f);
+  float2 x[4];
+  float w[4];
+#pragma unroll
+  for (int c = 0; c < 4; ++c) { x[c] = make_float2(threadIdx.x + c, c); w[c] = threadIdx.x - c; }
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      x[c] = __ffma2_rn(x[c], y, z);
+      w[c] = fmaf(w[c], y.x, z.y);
+    }
+  }
+  float s = 0; for (int c = 0; c < 4; ++c) s += x[c].x + x[c].y + w[c];
+  if (s == 1.2345f) out[0] = s;
+}
+
+// ---- the SDH distance stream: FADD2 with a broadcast scalar operand (a - p for two anchors)
+// then FFMA2 squares, as in run_chunk. Lane-ops = 2 per packed instruction.
+__global__ void k_dist(float* out, float p0) {
+  float2 a[4], s[4];
+#pragma unroll
+  for (int c = 0; c < 4; ++c) { a[c] = make_float2(threadIdx.x * 1e-3f + c, c * 0.5f); s[c] = make_float2(0.f, 0.f); }
+  float p = p0 + threadIdx.x * 1e-7f;
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      const float2 d = __fadd2_rn(a[c], make_float2(p, p));
+      s[c] = __ffma2_rn(d, d, s[c]);
+    }
+    p += 1e-6f;
+  }
+  float t = 0; for (int c = 0; c < 4; ++c) t += s[c].x + s[c].y;
+  if (t == 1.2345f) out[0] = t;
+}
+
 // ---- FP32 scalar FADD / packed FADD2 ----------------------------------------
 __global__ void k_fadd(float* out, float y0) {
   float y = y0 + threadIdx.x * 1e-9f;
@@ -211,6 +249,8 @@ int main() {
   double it = (double)ITERS * 8 * thr;
   rep("ffma", it, timeit([&] { k_ffma<<<blocks, threads>>>(dout, 0.999f, 0.001f); }));
   rep("ffma2_lanes", 2 * it, timeit([&] { k_ffma2<<<blocks, threads>>>(dout, 0.999f, 0.001f); }));
+  rep("ffma2_plus_ffma_lanes", (double)ITERS * 4 * 3 * thr, timeit([&] { k_mix<<<blocks, threads>>>(dout, 0.999f, 0.001f); }));
+  rep("fadd2_bcast_ffma2_lanes", (double)ITERS * 4 * 4 * thr, timeit([&] { k_dist<<<blocks, threads>>>(dout, 0.25f); }));
   rep("fadd", it, timeit([&] { k_fadd<<<blocks, threads>>>(dout, 0.001f); }));
   rep("fadd2_lanes", 2 * it, timeit([&] { k_fadd2<<<blocks, threads>>>(dout, 0.001f); }));
   rep("mufu_sqrt", it, timeit([&] { k_mufu<0><<<blocks, threads>>>(dout); }));

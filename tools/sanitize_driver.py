@@ -41,6 +41,9 @@ xb = torch.from_numpy(g.uniform(777, 4, 96)).cuda().to(torch.bfloat16)   # hd: C
 out.append(float(tbs.pairmatrix_hd(xb, 0.01).sum().item()))
 out.append(float(tbs.pairmatrix_hd(xb, 0.01, rows=(130, 419)).sum().item()))
 out.append(float(tbs.pairmatrix_hd(xb[:700], 0.01, kernel="dist").sum().item()))
+out.append(float(tbs.rdf(p, w, 64, 1.0).sum().item()))                 # RDF (NEXT-1)
+out.append(float(tbs.rdf(lat, 0.5, 64, 2197.0, lattice=True, rows=(5, 1500)).sum().item()))
+out.append(tbs.sdh(lat, 0.5, 64, lattice=True, validate=True).sum().item())   # TBS_VALIDATE
 big = torch.from_numpy(g.uniform(40000, 3)).cuda()                # main (non-small) tile config
 out.append(tbs.sdh(big, w, 64).sum().item())
 torch.cuda.synchronize()
