@@ -947,9 +947,155 @@ int staging(size_t bytes, void** out) {
   return TBS_OK;
 }
 
+// ---- small-problem plans for the simple entry points with host buffers -----------------
+// Launch latency, not arithmetic, bounds small problems (BASELINE configs[0], N = 4096: 8.4e6
+// pairs, a ~15 us pair kernel behind a loader and the host's launch calls). For host-buffer
+// calls with n <= kPlanMaxN the device work of a call (loader, pair kernel(s), flush) is
+// captured once per (operation, parameters, n, dim, device) into a CUDA graph over persistent
+// device buffers; later calls with the same key copy the points in, launch the graph and copy
+// the result out — one graph launch, no allocation. A few plans per thread (LRU); tbs_release()
+// drops the calling thread's plans.
+constexpr int64_t kPlanMaxN = 65536;
+constexpr int kPlanSlots = 8;
+struct PlanKey {
+  int op = -1;           // 0 SDH, 1 2PCF, 2 kernel density
+  int64_t n = 0;
+  int dim = 0;
+  float f = 0.f;         // bucket width / radius / gamma
+  long long i = 0;       // buckets
+  int dev = -1;
+  bool same(const PlanKey& o) const {
+    return op == o.op && n == o.n && dim == o.dim && memcmp(&f, &o.f, sizeof f) == 0 && i == o.i && dev == o.dev;
+  }
+};
+struct Plan {
+  PlanKey key;
+  cudaStream_t st = nullptr;
+  cudaGraphExec_t exec = nullptr;   // nullptr: capture failed, the plan runs its calls directly
+  unsigned char* dbuf = nullptr;    // [points | output]
+  size_t out_off = 0;
+  int kernels = 0;                  // kernel nodes in the graph (launch counter)
+  unsigned long long used = 0;
+  void destroy() {
+    if (exec) cudaGraphExecDestroy(exec);
+    if (dbuf) cudaFree(dbuf);
+    if (st) cudaStreamDestroy(st);
+    exec = nullptr;
+    dbuf = nullptr;
+    st = nullptr;
+  }
+};
+struct PlanCache {
+  Plan slot[kPlanSlots];
+  unsigned long long tick = 0;
+  ~PlanCache() { clear(); }
+  void clear() {
+    for (auto& p : slot) {
+      p.destroy();
+      p.key = PlanKey{};
+    }
+  }
+};
+PlanCache& plans() {
+  static thread_local PlanCache c;
+  return c;
+}
+
+// One host-buffer call through its plan (created, and its graph captured, on first use).
+template <class Fn>
+int run_plan(const PlanKey& key, const float* points, int pk, void* outp, int ok, size_t pbytes, size_t out_bytes,
+             Fn fn) {
+  PlanCache& pc = plans();
+  Plan* pl = nullptr;
+  for (auto& p : pc.slot)
+    if (p.key.same(key) && p.dbuf) pl = &p;
+  bool fresh = false;
+  if (!pl) {
+    pl = &pc.slot[0];
+    for (auto& p : pc.slot)
+      if (!p.dbuf || p.used < pl->used) pl = &p;     // an empty slot, else the least recently used
+    pl->destroy();
+    pl->key = key;
+    pl->out_off = (pbytes + 255) / 256 * 256;
+    TBS_CUDA(cudaStreamCreateWithFlags(&pl->st, cudaStreamNonBlocking));
+    cudaError_t e = cudaMalloc((void**)&pl->dbuf, pl->out_off + out_bytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      pl->destroy();
+      pl->key = PlanKey{};
+      return fail(TBS_ENOMEM, "plan buffers (%zu B): %s", pl->out_off + out_bytes, cudaGetErrorString(e));
+    }
+    fresh = true;
+  }
+  pl->used = ++pc.tick;
+  cudaStream_t st = pl->st;
+  tbs_args a{};
+  a.points = reinterpret_cast<const float*>(pl->dbuf);
+  a.n = key.n;
+  a.dim = key.dim;
+  a.row_begin = 0;
+  a.row_end = key.n;
+  a.stream = st;
+  void* dout = pl->dbuf + pl->out_off;
+  // pageable host buffers go through the pinned staging area: [points | output]
+  const size_t pin_in = pk == 1 ? 0 : pl->out_off, pin_out = ok == 1 ? 0 : out_bytes;
+  unsigned char* stage = nullptr;
+  if (pin_in + pin_out) {
+    void* sp = nullptr;
+    int rc = staging(pin_in + pin_out, &sp);
+    if (rc) return rc;
+    stage = static_cast<unsigned char*>(sp);
+  }
+  const void* src = points;
+  if (pin_in) {
+    memcpy(stage, points, pbytes);
+    src = stage;
+  }
+  void* dst = pin_out ? static_cast<void*>(stage + pin_in) : outp;
+  TBS_CUDA(cudaMemcpyAsync(pl->dbuf, src, pbytes, cudaMemcpyHostToDevice, st));
+  int rc = TBS_OK;
+  if (pl->exec) {
+    TBS_CUDA(cudaGraphLaunch(pl->exec, st));
+    g_launches.fetch_add((unsigned long long)pl->kernels);
+  } else {
+    rc = fn(&a, dout);            // first call of this plan (or capture unavailable): direct launches
+  }
+  if (!rc) TBS_CUDA(cudaMemcpyAsync(dst, dout, out_bytes, cudaMemcpyDeviceToHost, st));
+  TBS_CUDA(cudaStreamSynchronize(st));
+  if (rc) return rc;
+  if (pin_out) memcpy(outp, dst, out_bytes);
+  if (fresh) {
+    // capture the device work for the next calls (caches warmed by the call above); any failure
+    // leaves the plan on direct launches
+    cudaGraph_t g = nullptr;
+    if (cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal) == cudaSuccess) {
+      const int crc = fn(&a, dout);
+      const cudaError_t ce = cudaStreamEndCapture(st, &g);
+      if (crc == TBS_OK && ce == cudaSuccess && g) {
+        size_t nn = 0;
+        if (cudaGraphGetNodes(g, nullptr, &nn) == cudaSuccess && nn) {
+          std::vector<cudaGraphNode_t> nodes(nn);
+          cudaGraphGetNodes(g, nodes.data(), &nn);
+          for (auto nd : nodes) {
+            cudaGraphNodeType ty;
+            if (cudaGraphNodeGetType(nd, &ty) == cudaSuccess && ty == cudaGraphNodeTypeKernel) ++pl->kernels;
+          }
+        }
+        if (cudaGraphInstantiate(&pl->exec, g, 0) != cudaSuccess) pl->exec = nullptr;
+        g_launches.fetch_sub((unsigned long long)pl->kernels);   // captured, not launched
+      }
+      if (g) cudaGraphDestroy(g);
+    }
+    cudaGetLastError();   // a failed capture is not an error of this call
+    g_err.clear();
+  }
+  return TBS_OK;
+}
+
 // Run `fn(args_with_device_ptrs, dev_out)` for host or device buffers, synchronously.
 template <class Fn>
-int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_bytes, Fn fn) {
+int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_bytes, Fn fn,
+               PlanKey key = PlanKey{}) {
   if (n < 0 || n > TBS_MAX_N) return fail(TBS_EINVAL, "n out of range");
   if (dim < 1 || dim > 4) return fail(TBS_EINVAL, "dim out of range");
   if (!outp) return fail(TBS_EINVAL, "output is NULL");
@@ -973,6 +1119,12 @@ int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_b
     return rc;
   }
   const size_t pbytes = (size_t)n * dim * sizeof(float);
+  if (key.op >= 0 && n >= 2 && n <= kPlanMaxN && out_bytes <= (1u << 20)) {
+    if (cudaGetDevice(&key.dev) != cudaSuccess) return fail(TBS_ECUDA, "cudaGetDevice failed");
+    key.n = n;
+    key.dim = dim;
+    return run_plan(key, points, pk, outp, ok, pbytes, out_bytes, fn);
+  }
   // pageable buffers go through the pinned staging area: [points | output]
   size_t pin_in = pk == 1 ? 0 : (pbytes + 255) / 256 * 256;
   size_t pin_out = ok == 1 ? 0 : out_bytes;
@@ -1032,14 +1184,22 @@ int tbs_pairmatrix_ex(const tbs_args* args, tbs_kernel kernel, float* out) {
 int tbs_sdh(const float* points, int64_t n, int dim, float bucket_width, int nbuckets, uint64_t* hist) {
   g_err.clear();
   if (nbuckets < 1 || nbuckets > TBS_MAX_BUCKETS) return fail(TBS_EINVAL, "nbuckets out of range");
+  PlanKey key;
+  key.op = 0;
+  key.f = bucket_width;
+  key.i = nbuckets;
   return run_simple(points, n, dim, hist, (size_t)nbuckets * 8, [&](tbs_args* a, void* out) {
     return sdh_impl(a, bucket_width, nbuckets, (uint64_t*)out);
-  });
+  }, key);
 }
 
 int tbs_pcf(const float* points, int64_t n, float radius, uint64_t* count) {
   g_err.clear();
-  return run_simple(points, n, 3, count, 8, [&](tbs_args* a, void* out) { return pcf_impl(a, radius, (uint64_t*)out); });
+  PlanKey key;
+  key.op = 1;
+  key.f = radius;
+  return run_simple(points, n, 3, count, 8, [&](tbs_args* a, void* out) { return pcf_impl(a, radius, (uint64_t*)out); },
+                    key);
 }
 
 int tbs_pairmatrix(const float* points, int64_t n, tbs_kernel kernel, float* out) {
@@ -1056,7 +1216,10 @@ int tbs_kde_ex(const tbs_args* args, float gamma, double* sum) {
 
 int tbs_kde(const float* points, int64_t n, float gamma, double* sum) {
   g_err.clear();
-  return run_simple(points, n, 3, sum, 8, [&](tbs_args* a, void* out) { return kde_impl(a, gamma, (double*)out); });
+  PlanKey key;
+  key.op = 2;
+  key.f = gamma;
+  return run_simple(points, n, 3, sum, 8, [&](tbs_args* a, void* out) { return kde_impl(a, gamma, (double*)out); }, key);
 }
 
 int tbs_rdf_ex(const tbs_args* args, float bucket_width, int nbuckets, double volume, double* g) {
@@ -1238,6 +1401,7 @@ int tbs_peer_atomics_ok(const char* pci_bus_id, int* ok) {
 const char* tbs_last_error(void) { return g_err.c_str(); }
 
 void tbs_release(void) {
+  plans().clear();
   int dev;
   if (cudaGetDevice(&dev) != cudaSuccess) return;
   cudaMemPool_t pool;

@@ -150,16 +150,18 @@ __global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_
   }
 }
 
-// Upper bound on any pair distance from the loader's bounding box (+inf if unknown).
+// Upper bound on any pair distance from the loader's bounding box (+inf if unknown): fp32 with
+// a 1e-5 relative margin (the fp32 rounding of three squares, a sum and a square root is
+// < 1e-6), far below the two guard bins the no-clamp test keeps.
 __device__ __forceinline__ float bbox_diameter(const uint32_t* __restrict__ bbox, int D) {
   if (bbox == nullptr || (bbox[2 * D] & 1u) != 0u) return __int_as_float(0x7f800000);
-  double s = 0.0;
+  float s = 0.0f;
   for (int c = 0; c < D; ++c) {
     if (bbox[c] == 0u || bbox[D + c] == 0u) return __int_as_float(0x7f800000);
-    const double e = (double)ord2f(bbox[D + c]) - (double)ord2f(~bbox[c]);
-    s += e * e;
+    const float e = __fsub_ru(ord2f(bbox[D + c]), ord2f(~bbox[c]));
+    s = __fmaf_ru(e, e, s);
   }
-  return (float)(sqrt(s) * (1.0 + 1e-5));
+  return __fmul_ru(__fsqrt_ru(s), 1.00001f);
 }
 
 // ------------------------------------------------------------------------------------
@@ -413,20 +415,26 @@ struct SdhSmemOp {
     }
   }
 
-  // Sum the R replicas of each bin (segmented shuffle) and add to the global u64 output.
+  // Sum the R replicas of each bin and add to the global u64 output: one thread per bin reads
+  // its R words in a rotated order r = (j + (t >> (5 - LOG2R))) mod R, so at every step j the
+  // 32 lanes of a warp hit 32 distinct banks (bins t and t + 32/R differ in r), and zeroes them.
+  // Independent loads instead of a dependent shuffle chain per bin: the flush was ~40 % of a
+  // small (N = 4096) launch with the segmented-shuffle form (ncu source view, r02).
   __device__ void flush(unsigned char* smem) {
     uint32_t* h = reinterpret_cast<uint32_t*>(smem);
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int total = rows * R;
-    for (int e0 = warp * 32; e0 < total; e0 += kWarps * 32) {
-      const int e = e0 + lane;
+    const int t = threadIdx.x & 31;
+    const int rot = t >> (5 - LOG2R);
+    for (int k = threadIdx.x; k < rows; k += kThreads) {
       unsigned long long v = 0;
-      if (e < total) { v = h[e]; h[e] = 0u; }
-#pragma unroll
-      for (int off = 1; off < R; off <<= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
-      if ((lane & (R - 1)) == 0 && v != 0ull && e < total) {
-        const int k = (e >> LOG2R) + (RANGED ? klo : 0);
-        out->add(k < nb ? k : nb - 1, v);
+#pragma unroll 8
+      for (int j = 0; j < R; ++j) {
+        const int w = k * R + ((j + rot) & (R - 1));
+        v += h[w];
+        h[w] = 0u;
+      }
+      if (v != 0ull) {
+        const int kk = k + (RANGED ? klo : 0);
+        out->add(kk < nb ? kk : nb - 1, v);
       }
     }
   }
@@ -699,14 +707,16 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
   if (g.trace != nullptr && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
   op.out = &sink;   // (param space: the Op stays small, its copy lives in registers)
   op.init(smem);
-  const int variant = op.variant(bbox, D);
-  if (!((VSET >> variant) & 1)) return;   // CTA-uniform: another launch owns this variant
+  __shared__ int s_variant;
   if (tid == 0) {
+    s_variant = op.variant(bbox, D);   // kernel-uniform; one thread reads the box
     mbar_init(bar0, 1);
     mbar_init(bar1, 1);
     fence_mbar_init();
   }
   __syncthreads();
+  const int variant = s_variant;
+  if (!((VSET >> variant) & 1)) return;   // CTA-uniform: another launch owns this variant
 
   // Dynamic work distribution: CTAs grab chunks of g.chunk consecutive items from a global
   // counter, so every CTA runs until the whole triangle is done (the warp arbiter favours

@@ -41,7 +41,24 @@ def dev_path():
     torch.cuda.current_stream().synchronize()
 
 
+dp = pin.to(dev)
+dout = torch.empty(nb, dtype=torch.int64, device=dev)
+tiny = torch.zeros(1, device=dev)
+
+
+def dev_only():
+    tbs.sdh(dp, w, nb, out=dout)
+    torch.cuda.current_stream().synchronize()
+
+
+def floor_sync():
+    tiny.add_(1.0)
+    torch.cuda.current_stream().synchronize()
+
+
 out = dict(n=n, nb=nb,
+           us_one_torch_kernel_plus_sync=per_call(floor_sync),
+           us_device_call_plus_sync=per_call(dev_only),
            us_ctypes_roundtrip=per_call(lambda: tbs.lib().tbs_version(), 20000),
            us_host_entry_pinned_in=per_call(lambda: tbs.sdh_host(pin.numpy(), w, nb, out=hh)),
            us_host_entry_pageable_in=per_call(lambda: tbs.sdh_host(p, w, nb, out=hh)),
