@@ -246,12 +246,30 @@ int validate_common(const tbs_args* a, long long peer_words = 0) {
   return TBS_OK;
 }
 
+// Scratch provided by a small-problem plan (run_plan): its persistent device buffer holds the
+// SoA copy + box block, so the plan's captured graph has no allocation nodes. Thread-local,
+// set only around a plan's calls.
+struct PlanScratch {
+  unsigned char* base = nullptr;
+  size_t bytes = 0;
+};
+PlanScratch& plan_scratch() {
+  static thread_local PlanScratch s;
+  return s;
+}
+void release_soa(float* soa, cudaStream_t st) {
+  if (soa && reinterpret_cast<unsigned char*>(soa) != plan_scratch().base) cudaFreeAsync(soa, st);
+}
+
 // SoA copy of the points in stream-ordered scratch; the loader also zeroes `zero` words.
 // The allocation holds SoA [D][n_pad] followed by the 2D+1 bounding-box words.
 int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long long* zero, long long zero_words,
                 cudaStream_t st, uint32_t** bbox, float pad = 0.0f) {
   const size_t soa_bytes = (size_t)D * n_pad * sizeof(float);
-  TBS_CUDA(cudaMallocAsync((void**)soa, soa_bytes + 64, st));
+  if (plan_scratch().base && soa_bytes + 64 <= plan_scratch().bytes)
+    *soa = reinterpret_cast<float*>(plan_scratch().base);
+  else
+    TBS_CUDA(cudaMallocAsync((void**)soa, soa_bytes + 64, st));
   *bbox = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(*soa) + soa_bytes);
   // Small problems: one 1024-thread CTA writes the whole bounding-box block itself (no memset
   // launch before it: the small-problem path is latency-bound, BASELINE configs[0]).
@@ -540,7 +558,7 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
                       : sdh_dispatch<4, false>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee);
   }
   if (!rc && peers) rc = push_to_peers(a, acc, nb, st);
-  if (soa) cudaFreeAsync(soa, st);
+  release_soa(soa, st);
   if (part) cudaFreeAsync(part, st);
   if (acc) cudaFreeAsync(acc, st);
   return rc;
@@ -583,7 +601,7 @@ int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
                   : launch_pair<PcfOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink);
   }
   if (!rc && peers) rc = push_to_peers(a, acc, 1, st);
-  if (soa) cudaFreeAsync(soa, st);
+  release_soa(soa, st);
   return rc;
 }
 
@@ -618,7 +636,7 @@ int kde_impl(const tbs_args* a, float gamma, double* sum) {
       rc = D == 3 ? launch_pair<KdeOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee)
                   : launch_pair<KdeOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee);
   }
-  if (soa) cudaFreeAsync(soa, st);
+  release_soa(soa, st);
   return rc;
 }
 
@@ -699,7 +717,7 @@ int pairmatrix_impl(const tbs_args* a, tbs_kernel k, float* out) {
               : k.type == 1 ? matrix_launch<1, 4>(a, soa, n_pad, cexp, out, st)
                             : matrix_launch<2, 4>(a, soa, n_pad, cexp, out, st);
   }
-  if (soa) cudaFreeAsync(soa, st);
+  release_soa(soa, st);
   return rc;
 }
 
@@ -896,7 +914,7 @@ int knn_impl(const tbs_args* a, int k, int32_t* idx, float* dist) {
               : k <= 16 ? knn_launch<16, 2, 4>(dev, a, soa, n_pad, k, idx, dist, st)
                         : knn_launch<32, 2, 4>(dev, a, soa, n_pad, k, idx, dist, st);
   }
-  if (soa) cudaFreeAsync(soa, st);
+  release_soa(soa, st);
   return rc;
 }
 
@@ -974,6 +992,7 @@ struct Plan {
   cudaGraphExec_t exec = nullptr;   // nullptr: capture failed, the plan runs its calls directly
   unsigned char* dbuf = nullptr;    // [points | output]
   size_t out_off = 0;
+  size_t scr_off = 0, scr_bytes = 0;  // the loader's SoA + box scratch inside dbuf
   int kernels = 0;                  // kernel nodes in the graph (launch counter)
   unsigned long long used = 0;
   void destroy() {
@@ -1017,13 +1036,15 @@ int run_plan(const PlanKey& key, const float* points, int pk, void* outp, int ok
     pl->destroy();
     pl->key = key;
     pl->out_off = (pbytes + 255) / 256 * 256;
+    pl->scr_off = (pl->out_off + out_bytes + 255) / 256 * 256;
+    pl->scr_bytes = (size_t)4 * pad_rows(key.n) * sizeof(float) + 64;   // SoA [D <= 4][n_pad] + box block
     TBS_CUDA(cudaStreamCreateWithFlags(&pl->st, cudaStreamNonBlocking));
-    cudaError_t e = cudaMalloc((void**)&pl->dbuf, pl->out_off + out_bytes);
+    cudaError_t e = cudaMalloc((void**)&pl->dbuf, pl->scr_off + pl->scr_bytes);
     if (e != cudaSuccess) {
       cudaGetLastError();
       pl->destroy();
       pl->key = PlanKey{};
-      return fail(TBS_ENOMEM, "plan buffers (%zu B): %s", pl->out_off + out_bytes, cudaGetErrorString(e));
+      return fail(TBS_ENOMEM, "plan buffers (%zu B): %s", pl->scr_off + pl->scr_bytes, cudaGetErrorString(e));
     }
     fresh = true;
   }
@@ -1054,6 +1075,10 @@ int run_plan(const PlanKey& key, const float* points, int pk, void* outp, int ok
   void* dst = pin_out ? static_cast<void*>(stage + pin_in) : outp;
   TBS_CUDA(cudaMemcpyAsync(pl->dbuf, src, pbytes, cudaMemcpyHostToDevice, st));
   int rc = TBS_OK;
+  struct ScratchScope {          // the plan's scratch for the loader while fn runs
+    explicit ScratchScope(unsigned char* p, size_t b) { plan_scratch().base = p; plan_scratch().bytes = b; }
+    ~ScratchScope() { plan_scratch() = PlanScratch{}; }
+  } scope(pl->dbuf + pl->scr_off, pl->scr_bytes);
   if (pl->exec) {
     TBS_CUDA(cudaGraphLaunch(pl->exec, st));
     g_launches.fetch_add((unsigned long long)pl->kernels);

@@ -420,6 +420,9 @@ struct SdhSmemOp {
   // 32 lanes of a warp hit 32 distinct banks (bins t and t + 32/R differ in r), and zeroes them.
   // Independent loads instead of a dependent shuffle chain per bin: the flush was ~40 % of a
   // small (N = 4096) launch with the segmented-shuffle form (ncu source view, r02).
+  // (Used for the final flush only: inside the item loop, the divergent per-thread loop cost the
+  // hot loop its uniform-datapath addressing and 7 % at N = 1M on B200 — the mid-kernel
+  // overflow flush keeps the warp-synchronous form below.)
   __device__ void flush(unsigned char* smem) {
     uint32_t* h = reinterpret_cast<uint32_t*>(smem);
     const int t = threadIdx.x & 31;
@@ -438,10 +441,28 @@ struct SdhSmemOp {
       }
     }
   }
+  // Mid-kernel overflow flush: segmented shuffle-sum of each bin's R replicas (warp-uniform
+  // loop, so the item loop around it keeps its uniform registers).
+  __device__ void flush_in_loop(unsigned char* smem) {
+    uint32_t* h = reinterpret_cast<uint32_t*>(smem);
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int total = rows * R;
+    for (int e0 = warp * 32; e0 < total; e0 += kWarps * 32) {
+      const int e = e0 + lane;
+      unsigned long long v = 0;
+      if (e < total) { v = h[e]; h[e] = 0u; }
+#pragma unroll
+      for (int off = 1; off < R; off <<= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+      if ((lane & (R - 1)) == 0 && v != 0ull && e < total) {
+        const int k = (e >> LOG2R) + (RANGED ? klo : 0);
+        out->add(k < nb ? k : nb - 1, v);
+      }
+    }
+  }
   __device__ __forceinline__ void after_group() {}
   __device__ __forceinline__ void after_item(unsigned char* smem, int& since) {
     if (++since >= flush_every) {
-      flush(smem);
+      flush_in_loop(smem);
       __syncthreads();
       since = 0;
     }
@@ -707,16 +728,16 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
   if (g.trace != nullptr && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_start));
   op.out = &sink;   // (param space: the Op stays small, its copy lives in registers)
   op.init(smem);
-  __shared__ int s_variant;
+  // kernel-uniform variant, computed by every thread from the same box (provably uniform: the
+  // item loop's addressing stays on the uniform datapath)
+  const int variant = op.variant(bbox, D);
+  if (!((VSET >> variant) & 1)) return;   // CTA-uniform: another launch owns this variant
   if (tid == 0) {
-    s_variant = op.variant(bbox, D);   // kernel-uniform; one thread reads the box
     mbar_init(bar0, 1);
     mbar_init(bar1, 1);
     fence_mbar_init();
   }
   __syncthreads();
-  const int variant = s_variant;
-  if (!((VSET >> variant) & 1)) return;   // CTA-uniform: another launch owns this variant
 
   // Dynamic work distribution: CTAs grab chunks of g.chunk consecutive items from a global
   // counter, so every CTA runs until the whole triangle is done (the warp arbiter favours
