@@ -273,13 +273,19 @@ int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long 
   *bbox = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(*soa) + soa_bytes);
   // Small problems: one 1024-thread CTA writes the whole bounding-box block itself (no memset
   // launch before it: the small-problem path is latency-bound, BASELINE configs[0]).
-  const bool one = n_pad <= 16384 && zero_words <= (1 << 16);
-  if (!one) TBS_CUDA(cudaMemsetAsync(*bbox, 0, 64, st));
-  const int threads = one ? 1024 : 256;
-  long long blocks = one ? 1 : std::min<long long>((n_pad + threads - 1) / threads, 148ll * 16);
-  blocks = std::max<long long>(blocks, 1);
-  soa_loader<<<(unsigned)blocks, threads, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, D, pad, *soa, zero,
-                                                   zero_words, *bbox);
+  if (n_pad <= kSmallLoad && zero_words <= (1 << 16)) {
+    if (D == 3)
+      soa_loader_small<3><<<1, 1024, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, pad, *soa, zero, (int)zero_words, *bbox);
+    else
+      soa_loader_small<4><<<1, 1024, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, pad, *soa, zero, (int)zero_words, *bbox);
+  } else {
+    TBS_CUDA(cudaMemsetAsync(*bbox, 0, 64, st));
+    const int threads = 256;
+    long long blocks = std::min<long long>((n_pad + threads - 1) / threads, 148ll * 16);
+    blocks = std::max<long long>(blocks, 1);
+    soa_loader<<<(unsigned)blocks, threads, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, D, pad, *soa, zero,
+                                                     zero_words, *bbox);
+  }
   TBS_CUDA(cudaGetLastError());
   g_launches.fetch_add(1);
   return TBS_OK;

@@ -119,15 +119,6 @@ __global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_
   }
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < zero_words; i += stride) zero[i] = 0ull;
   if (bbox) {
-    // One-CTA launch (small problems): reduce in shared memory and write the whole 64-byte
-    // block (box, flags, zeroed work-queue counter), so the caller needs no memset before it.
-    __shared__ uint32_t sb[16];
-    const bool one = gridDim.x == 1;
-    if (one) {
-      if (threadIdx.x < 16) sb[threadIdx.x] = 0u;
-      __syncthreads();
-    }
-    uint32_t* dst = one ? sb : bbox;
     for (int c = 0; c < D; ++c) {
       uint32_t a = lo[c], b = hi[c];
 #pragma unroll
@@ -136,18 +127,65 @@ __global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_
         b = max(b, __shfl_xor_sync(0xffffffffu, b, off));
       }
       if ((threadIdx.x & 31) == 0) {
-        if (a) atomicMax(dst + c, a);
-        if (b) atomicMax(dst + D + c, b);
+        if (a) atomicMax(bbox + c, a);
+        if (b) atomicMax(bbox + D + c, b);
       }
     }
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) bad |= __shfl_xor_sync(0xffffffffu, bad, off);
-    if ((threadIdx.x & 31) == 0 && bad) atomicOr(dst + 2 * D, bad);
-    if (one) {
-      __syncthreads();
-      if (threadIdx.x < 16) bbox[threadIdx.x] = sb[threadIdx.x];
+    if ((threadIdx.x & 31) == 0 && bad) atomicOr(bbox + 2 * D, bad);
+  }
+}
+
+// The same for small problems (n_pad <= kSmallLoad): ONE 1024-thread CTA, D a template
+// argument, 32-bit indices, reduction in shared memory, and the whole 64-byte box block
+// written at the end, so the caller needs no memset before it (the small-problem path is
+// latency-bound, BASELINE configs[0]; the general loader took 9.8 us there, ncu r02).
+constexpr int kSmallLoad = 16384;
+template <int D>
+__global__ void __launch_bounds__(1024) soa_loader_small(const float* __restrict__ pts, int n, int dim, int n_pad, float pad,
+                                                          float* __restrict__ soa, unsigned long long* __restrict__ zero,
+                                                          int zero_words, uint32_t* __restrict__ bbox) {
+  __shared__ uint32_t sb[16];
+  if (threadIdx.x < 16) sb[threadIdx.x] = 0u;
+  uint32_t lo[D], hi[D], bad = 0u;
+#pragma unroll
+  for (int c = 0; c < D; ++c) lo[c] = hi[c] = 0u;
+#pragma unroll 4
+  for (int i = threadIdx.x; i < n_pad; i += 1024) {
+#pragma unroll
+    for (int c = 0; c < D; ++c) {
+      float v = pad;
+      if (i < n) {
+        v = c < dim ? __ldg(pts + i * dim + c) : 0.0f;
+        const uint32_t o = f2ord(v);
+        lo[c] = max(lo[c], ~o);
+        hi[c] = max(hi[c], o);
+        bad |= (isfinite(v) ? 0u : 1u) | (v == rintf(v) ? 0u : 2u);
+      }
+      soa[c * n_pad + i] = v;
     }
   }
+  for (int i = threadIdx.x; i < zero_words; i += 1024) zero[i] = 0ull;
+  __syncthreads();
+#pragma unroll
+  for (int c = 0; c < D; ++c) {
+    uint32_t a = lo[c], b = hi[c];
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      a = max(a, __shfl_xor_sync(0xffffffffu, a, off));
+      b = max(b, __shfl_xor_sync(0xffffffffu, b, off));
+    }
+    if ((threadIdx.x & 31) == 0) {
+      if (a) atomicMax(sb + c, a);
+      if (b) atomicMax(sb + D + c, b);
+    }
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) bad |= __shfl_xor_sync(0xffffffffu, bad, off);
+  if ((threadIdx.x & 31) == 0 && bad) atomicOr(sb + 2 * D, bad);
+  __syncthreads();
+  if (threadIdx.x < 16) bbox[threadIdx.x] = sb[threadIdx.x];
 }
 
 // Upper bound on any pair distance from the loader's bounding box (+inf if unknown): fp32 with

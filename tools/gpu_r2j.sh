@@ -1,0 +1,9 @@
+set -x
+mkdir -p gpurun_out/r2j
+ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/r2j/c1_launches.csv python tools/c1_probe.py > gpurun_out/r2j/c1.log 2>&1
+timeout 300 python bench.py --no-cpu-baseline --workload sdh_uniform_4k --steps 50 > gpurun_out/r2j/c1_graph.json 2>&1
+timeout 300 python bench.py --no-cpu-baseline --workload sdh_uniform_4k --steps 50 --graph off > gpurun_out/r2j/c1_nograph.json 2>&1
+timeout 300 python tools/c1_e2e.py > gpurun_out/r2j/c1_e2e.json 2>&1
+timeout 600 python bench.py --no-cpu-baseline > gpurun_out/r2j/bench_1m.json 2>&1
+timeout 1500 python -m pytest tests/test_gpu_parity.py tests/test_gpu_fused.py -m gpu -x -q > gpurun_out/r2j/pytest.txt 2>&1
+tail -2 gpurun_out/r2j/pytest.txt
