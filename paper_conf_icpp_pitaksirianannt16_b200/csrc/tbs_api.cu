@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <atomic>
 #include <cmath>
 #include <cstdarg>
@@ -220,6 +221,36 @@ int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op
             "span %.3f ms, latest start %.3f ms\n", grid, occ, mn, mx, dmin * 1e-6, dsum / grid * 1e-6, dmax * 1e-6,
             (t1 - t0) * 1e-6, late * 1e-6);
   }
+  return TBS_OK;
+}
+
+// Small problems (fewer items than small_items_per_sm() per SM, n <= kSmallLoad): the fused
+// one-item-per-CTA kernel reading the caller's AoS points (no loader launch, no SoA scratch).
+bool small_fused(const Device& dev, const tbs_args* a) {
+  if (a->n > kSmallLoad || (a->flags & TBS_VALIDATE)) return false;
+  return make_geom(a->n, a->row_begin, a->row_end, SdhCfg::TA, SdhCfg::TP).items <
+         (long long)small_items_per_sm() * dev.sms;
+}
+
+template <class Op, int D, int V>
+int launch_small(const Device& dev, const tbs_args* a, const Op& op, cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee,
+                 const OutSink& sink) {
+  using C = SmallCfg;
+  auto kern = pair_kernel_small<Op, D, C, V>;
+  const Geom g = make_geom(a->n, a->row_begin, a->row_end, C::TA, C::TP);
+  const long long smem = ((op.smem_bytes() + 127) & ~127ll) + (long long)D * C::TP * 4 + 16;
+  if (smem > dev.smem_optin) return fail(TBS_EUNSUPPORTED, "small pair kernel needs %lld B smem", smem);
+  struct AttrCache { int dev = -1; long long smem = -1; };
+  static thread_local AttrCache cache;
+  if (cache.dev != dev.id || cache.smem < smem) {
+    TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    cache = AttrCache{dev.id, smem};
+  }
+  if (eb) TBS_CUDA(cudaEventRecord(eb, st));
+  kern<<<(unsigned)g.items, kThreads, (size_t)smem, st>>>(a->points, a->dim, g, op, sink);
+  TBS_CUDA(cudaGetLastError());
+  g_launches.fetch_add(1);
+  if (ee) TBS_CUDA(cudaEventRecord(ee, st));
   return TBS_OK;
 }
 
@@ -540,6 +571,21 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   if (a->flags & TBS_HIST_FORCE_GLOBAL) pl = SdhPlan{lattice, true, 0};
 
   const int D = a->dim <= 3 ? 3 : 4;
+  if (!lattice && !pl.global && pl.passes == 1 && pl.log2r == 5 && small_fused(dev, a)) {
+    // small problem: zero the output, one fused launch (clamp variant: no bounding box)
+    SdhSmemOp<5, false> op{};
+    op.nb = nb;
+    op.rows = nb + kGuard;
+    op.inv_w = (float)(1.0 / (double)w);
+    op.flush_every = (int)std::max<long long>(1, 0xffffffffll / ((long long)kWarps * SmallCfg::KA * SmallCfg::TP) - 1);
+    TBS_CUDA(cudaMemsetAsync(h, 0, (size_t)nb * 8, st));
+    cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
+    rc = D == 3 ? launch_small<SdhSmemOp<5, false>, 3, 1>(dev, a, op, st, eb, ee, sink)
+                : launch_small<SdhSmemOp<5, false>, 4, 1>(dev, a, op, st, eb, ee, sink);
+    if (!rc && peers) rc = push_to_peers(a, acc, nb, st);
+    if (acc) cudaFreeAsync(acc, st);
+    return rc;
+  }
   const int n_pad = pad_rows(a->n);
   int G = 0;
   unsigned long long* part = nullptr;
@@ -585,6 +631,14 @@ int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
     return TBS_OK;
   }
   const int D = a->dim <= 3 ? 3 : 4;
+  if (!peers && small_fused(dev, a)) {
+    PcfOp op{};
+    op.r2 = (float)((double)r * (double)r);
+    TBS_CUDA(cudaMemsetAsync(c, 0, 8, st));
+    cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
+    return D == 3 ? launch_small<PcfOp, 3, 0>(dev, a, op, st, eb, ee, local_sink(c))
+                  : launch_small<PcfOp, 4, 0>(dev, a, op, st, eb, ee, local_sink(c));
+  }
   float* soa = nullptr;
   uint32_t* bbox = nullptr;
   rc = load_points(a, D, pad_rows(a->n), &soa, peers ? nullptr : c, peers ? 0 : 1, st, &bbox);
@@ -624,6 +678,15 @@ int kde_impl(const tbs_args* a, float gamma, double* sum) {
     return TBS_OK;
   }
   const int D = a->dim <= 3 ? 3 : 4;
+  if (small_fused(dev, a)) {
+    KdeOp op{};
+    op.c = (float)(-(double)gamma * 1.4426950408889634);
+    op.sum = sum;
+    TBS_CUDA(cudaMemsetAsync(sum, 0, 8, st));
+    cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
+    return D == 3 ? launch_small<KdeOp, 3, 0>(dev, a, op, st, eb, ee, OutSink{})
+                  : launch_small<KdeOp, 4, 0>(dev, a, op, st, eb, ee, OutSink{});
+  }
   float* soa = nullptr;
   uint32_t* bbox = nullptr;
   rc = load_points(a, D, pad_rows(a->n), &soa, reinterpret_cast<unsigned long long*>(sum), 1, st, &bbox);
@@ -1026,6 +1089,32 @@ PlanCache& plans() {
   return c;
 }
 
+// TBS_HOST_TRACE=1 (experiments): average host microseconds of the plan path's phases, printed
+// to stderr every 1000 plan calls.
+struct HostTrace {
+  bool on = getenv("TBS_HOST_TRACE") != nullptr;
+  double acc[8] = {0};
+  long calls = 0;
+  std::chrono::steady_clock::time_point t0;
+  void start() { if (on) t0 = std::chrono::steady_clock::now(); }
+  void mark(int k) {
+    if (!on) return;
+    const auto t = std::chrono::steady_clock::now();
+    acc[k] += std::chrono::duration<double, std::micro>(t - t0).count();
+    t0 = t;
+  }
+  void done() {
+    if (!on || ++calls % 1000) return;
+    fprintf(stderr, "[tbs host] per plan call (us): stage-in %.2f  H2D-enqueue %.2f  launch %.2f  D2H-enqueue %.2f  "
+            "sync %.2f  stage-out %.2f\n", acc[0] / calls, acc[1] / calls, acc[2] / calls, acc[3] / calls, acc[4] / calls,
+            acc[5] / calls);
+  }
+};
+HostTrace& host_trace() {
+  static thread_local HostTrace t;
+  return t;
+}
+
 // One host-buffer call through its plan (created, and its graph captured, on first use).
 template <class Fn>
 int run_plan(const PlanKey& key, const float* points, int pk, void* outp, int ok, size_t pbytes, size_t out_bytes,
@@ -1073,13 +1162,17 @@ int run_plan(const PlanKey& key, const float* points, int pk, void* outp, int ok
     if (rc) return rc;
     stage = static_cast<unsigned char*>(sp);
   }
+  HostTrace& ht = host_trace();
+  ht.start();
   const void* src = points;
   if (pin_in) {
     memcpy(stage, points, pbytes);
     src = stage;
   }
+  ht.mark(0);
   void* dst = pin_out ? static_cast<void*>(stage + pin_in) : outp;
   TBS_CUDA(cudaMemcpyAsync(pl->dbuf, src, pbytes, cudaMemcpyHostToDevice, st));
+  ht.mark(1);
   int rc = TBS_OK;
   struct ScratchScope {          // the plan's scratch for the loader while fn runs
     explicit ScratchScope(unsigned char* p, size_t b) { plan_scratch().base = p; plan_scratch().bytes = b; }
@@ -1091,10 +1184,15 @@ int run_plan(const PlanKey& key, const float* points, int pk, void* outp, int ok
   } else {
     rc = fn(&a, dout);            // first call of this plan (or capture unavailable): direct launches
   }
+  ht.mark(2);
   if (!rc) TBS_CUDA(cudaMemcpyAsync(dst, dout, out_bytes, cudaMemcpyDeviceToHost, st));
+  ht.mark(3);
   TBS_CUDA(cudaStreamSynchronize(st));
+  ht.mark(4);
   if (rc) return rc;
   if (pin_out) memcpy(outp, dst, out_bytes);
+  ht.mark(5);
+  if (!fresh) ht.done();
   if (fresh) {
     // capture the device work for the next calls (caches warmed by the call above); any failure
     // leaves the plan on direct launches

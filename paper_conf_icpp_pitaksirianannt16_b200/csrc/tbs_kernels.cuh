@@ -909,6 +909,48 @@ __global__ void push_peers(const unsigned long long* __restrict__ acc, int words
   out.fence();
 }
 
+// Small problems (BASELINE configs[0], N = 4096): one work item per CTA and the loader fused
+// in. Each CTA reads its anchors and its partner chunk straight from the caller's AoS points
+// (the chunk, D x TP floats, is one contiguous AoS span, transposed into the shared-memory
+// SoA layout run_chunk reads), so the call is one memset of the output plus this launch
+// instead of a loader launch plus the pair kernel (the loader was ~7 us of a ~20 us step).
+// No bounding box exists here: float SDH takes the clamp variant V.
+template <class Op, int D, class C, int V>
+__global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel_small(const float* __restrict__ pts, int dim, Geom g,
+                                                                  Op op, const __grid_constant__ OutSink sink) {
+  unsigned char* smem = tbs_smem;
+  const long long hbytes = (op.smem_bytes() + 127) & ~127ll;
+  float* B = reinterpret_cast<float*>(smem + hbytes);
+  const int tid = threadIdx.x;
+  op.out = &sink;
+  op.init(smem);
+  int I, J;
+  item_to_tile(g, (long long)blockIdx.x, I, J);
+  const int p0 = J * C::TP;
+  for (int p = tid; p < C::TP; p += kThreads) {
+    const long long j = p0 + p;
+#pragma unroll
+    for (int c = 0; c < D; ++c) B[c * C::TP + p] = (j < g.n && c < dim) ? __ldg(pts + j * dim + c) : 0.0f;
+  }
+  float2 na[D][C::KA / 2];
+#pragma unroll
+  for (int k = 0; k < C::KA; ++k) {
+    const long long a = (long long)I * C::TA + k * kThreads + tid;
+#pragma unroll
+    for (int c = 0; c < D; ++c) {
+      const float v = (a < g.n && c < dim) ? -__ldg(pts + a * dim + c) : 0.0f;
+      if (k & 1) na[c][k >> 1].y = v; else na[c][k >> 1].x = v;
+    }
+  }
+  __syncthreads();
+  const int cnt = min(C::TP, g.n - p0);
+  const bool fast = (I * C::TA >= g.rb) && ((I + 1) * C::TA <= g.re) && (p0 >= (I + 1) * C::TA) && (cnt == C::TP);
+  if (fast) run_chunk<Op, D, C, false, V>(op, B, na, g, I, p0, cnt);
+  else run_chunk<Op, D, C, true, V>(op, B, na, g, I, p0, cnt);
+  __syncthreads();
+  op.finish(smem);
+}
+
 // Sum G partial global copies into the output (one thread per bin, the paper's
 // reduction kernel K13, L778-782).
 __global__ void reduce_partials(const unsigned long long* __restrict__ part, int G, int nb,

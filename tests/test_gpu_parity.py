@@ -287,6 +287,9 @@ def test_host_pointer_entry_points(tbs):
 def test_launch_counter_moves(tbs):
     before = tbs.launch_count()
     sdh_gpu(tbs, g.uniform(3000, 1), 0.05, 32)
+    assert tbs.launch_count() >= before + 1           # small problem: one fused launch
+    before = tbs.launch_count()
+    sdh_gpu(tbs, g.uniform(40000, 1), 0.05, 32)
     assert tbs.launch_count() >= before + 2           # loader + pair kernel
 
 
