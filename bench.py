@@ -546,15 +546,24 @@ def main():
             hh = np.zeros(nb if op == "sdh" else 1, np.uint64)
             kh = np.zeros(1, np.float64)
 
+            # the C-ABI host-buffer entry points (tbs_sdh / tbs_pcf / tbs_kde: the north star's
+            # signatures) called directly, arguments marshalled once; status checked every call
+            L, pptr = tbs.lib(), ph.numpy().ctypes.data
+            ch = np.zeros(1, np.uint64)
+            cw, cg, cr = ctypes.c_float(w), ctypes.c_float(params.get("gamma", 0.0)), ctypes.c_float(params.get("r", 0.0))
+
             def e2e_step():
                 if op == "sdh":
-                    tbs.sdh_host(ph.numpy(), w, nb, out=hh)
+                    rc = L.tbs_sdh(pptr, n, 3, cw, nb, hh.ctypes.data)
                 elif op == "kde":
-                    tbs.lib().tbs_kde(ph.numpy().ctypes.data, n, ctypes.c_float(params["gamma"]), kh.ctypes.data)
+                    rc = L.tbs_kde(pptr, n, cg, kh.ctypes.data)
                 elif op == "knn":
                     tbs.knn_host(ph.numpy(), params["k"])
+                    rc = 0
                 else:
-                    tbs.pcf_host(ph.numpy(), params["r"])
+                    rc = L.tbs_pcf(pptr, n, cr, ch.ctypes.data)
+                if rc:
+                    raise tbs.TbsError(f"e2e call: status {rc}: {tbs.last_error()}")
         else:
             res_h = torch.empty((out[1] if op == "knn" else out).shape, dtype=(out[1] if op == "knn" else out).dtype).pin_memory()
 

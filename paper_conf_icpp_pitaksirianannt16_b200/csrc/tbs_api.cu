@@ -232,6 +232,18 @@ bool small_fused(const Device& dev, const tbs_args* a) {
          (long long)small_items_per_sm() * dev.sms;
 }
 
+// A host-buffer call's request to the small fused path (thread-local, set by run_simple around
+// its call): the output and ticket are already zeroed; the kernel's last CTA writes the result
+// to mapped host memory. `taken` reports whether the path consumed it.
+struct SmallWriteBack {
+  WriteBack wb;
+  bool active = false, taken = false;
+};
+SmallWriteBack& small_wb() {
+  static thread_local SmallWriteBack w;
+  return w;
+}
+
 template <class Op, int D, int V>
 int launch_small(const Device& dev, const tbs_args* a, const Op& op, cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee,
                  const OutSink& sink) {
@@ -247,7 +259,12 @@ int launch_small(const Device& dev, const tbs_args* a, const Op& op, cudaStream_
     cache = AttrCache{dev.id, smem};
   }
   if (eb) TBS_CUDA(cudaEventRecord(eb, st));
-  kern<<<(unsigned)g.items, kThreads, (size_t)smem, st>>>(a->points, a->dim, g, op, sink);
+  WriteBack wb{};
+  if (small_wb().active) {
+    wb = small_wb().wb;
+    small_wb().taken = true;
+  }
+  kern<<<(unsigned)g.items, kThreads, (size_t)smem, st>>>(a->points, a->dim, g, op, sink, wb);
   TBS_CUDA(cudaGetLastError());
   g_launches.fetch_add(1);
   if (ee) TBS_CUDA(cudaEventRecord(ee, st));
@@ -277,19 +294,8 @@ int validate_common(const tbs_args* a, long long peer_words = 0) {
   return TBS_OK;
 }
 
-// Scratch provided by a small-problem plan (run_plan): its persistent device buffer holds the
-// SoA copy + box block, so the plan's captured graph has no allocation nodes. Thread-local,
-// set only around a plan's calls.
-struct PlanScratch {
-  unsigned char* base = nullptr;
-  size_t bytes = 0;
-};
-PlanScratch& plan_scratch() {
-  static thread_local PlanScratch s;
-  return s;
-}
 void release_soa(float* soa, cudaStream_t st) {
-  if (soa && reinterpret_cast<unsigned char*>(soa) != plan_scratch().base) cudaFreeAsync(soa, st);
+  if (soa) cudaFreeAsync(soa, st);
 }
 
 // SoA copy of the points in stream-ordered scratch; the loader also zeroes `zero` words.
@@ -297,10 +303,7 @@ void release_soa(float* soa, cudaStream_t st) {
 int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long long* zero, long long zero_words,
                 cudaStream_t st, uint32_t** bbox, float pad = 0.0f) {
   const size_t soa_bytes = (size_t)D * n_pad * sizeof(float);
-  if (plan_scratch().base && soa_bytes + 64 <= plan_scratch().bytes)
-    *soa = reinterpret_cast<float*>(plan_scratch().base);
-  else
-    TBS_CUDA(cudaMallocAsync((void**)soa, soa_bytes + 64, st));
+  TBS_CUDA(cudaMallocAsync((void**)soa, soa_bytes + 64, st));
   *bbox = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(*soa) + soa_bytes);
   // Small problems: one 1024-thread CTA writes the whole bounding-box block itself (no memset
   // launch before it: the small-problem path is latency-bound, BASELINE configs[0]).
@@ -578,7 +581,7 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
     op.rows = nb + kGuard;
     op.inv_w = (float)(1.0 / (double)w);
     op.flush_every = (int)std::max<long long>(1, 0xffffffffll / ((long long)kWarps * SmallCfg::KA * SmallCfg::TP) - 1);
-    TBS_CUDA(cudaMemsetAsync(h, 0, (size_t)nb * 8, st));
+    if (!small_wb().active || peers) TBS_CUDA(cudaMemsetAsync(h, 0, (size_t)nb * 8, st));
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
     rc = D == 3 ? launch_small<SdhSmemOp<5, false>, 3, 1>(dev, a, op, st, eb, ee, sink)
                 : launch_small<SdhSmemOp<5, false>, 4, 1>(dev, a, op, st, eb, ee, sink);
@@ -634,7 +637,7 @@ int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
   if (!peers && small_fused(dev, a)) {
     PcfOp op{};
     op.r2 = (float)((double)r * (double)r);
-    TBS_CUDA(cudaMemsetAsync(c, 0, 8, st));
+    if (!small_wb().active) TBS_CUDA(cudaMemsetAsync(c, 0, 8, st));
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
     return D == 3 ? launch_small<PcfOp, 3, 0>(dev, a, op, st, eb, ee, local_sink(c))
                   : launch_small<PcfOp, 4, 0>(dev, a, op, st, eb, ee, local_sink(c));
@@ -682,7 +685,7 @@ int kde_impl(const tbs_args* a, float gamma, double* sum) {
     KdeOp op{};
     op.c = (float)(-(double)gamma * 1.4426950408889634);
     op.sum = sum;
-    TBS_CUDA(cudaMemsetAsync(sum, 0, 8, st));
+    if (!small_wb().active) TBS_CUDA(cudaMemsetAsync(sum, 0, 8, st));
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
     return D == 3 ? launch_small<KdeOp, 3, 0>(dev, a, op, st, eb, ee, OutSink{})
                   : launch_small<KdeOp, 4, 0>(dev, a, op, st, eb, ee, OutSink{});
@@ -1034,197 +1037,10 @@ int staging(size_t bytes, void** out) {
   return TBS_OK;
 }
 
-// ---- small-problem plans for the simple entry points with host buffers -----------------
-// Launch latency, not arithmetic, bounds small problems (BASELINE configs[0], N = 4096: 8.4e6
-// pairs, a ~15 us pair kernel behind a loader and the host's launch calls). For host-buffer
-// calls with n <= kPlanMaxN the device work of a call (loader, pair kernel(s), flush) is
-// captured once per (operation, parameters, n, dim, device) into a CUDA graph over persistent
-// device buffers; later calls with the same key copy the points in, launch the graph and copy
-// the result out — one graph launch, no allocation. A few plans per thread (LRU); tbs_release()
-// drops the calling thread's plans.
-constexpr int64_t kPlanMaxN = 65536;
-constexpr int kPlanSlots = 8;
-struct PlanKey {
-  int op = -1;           // 0 SDH, 1 2PCF, 2 kernel density
-  int64_t n = 0;
-  int dim = 0;
-  float f = 0.f;         // bucket width / radius / gamma
-  long long i = 0;       // buckets
-  int dev = -1;
-  bool same(const PlanKey& o) const {
-    return op == o.op && n == o.n && dim == o.dim && memcmp(&f, &o.f, sizeof f) == 0 && i == o.i && dev == o.dev;
-  }
-};
-struct Plan {
-  PlanKey key;
-  cudaStream_t st = nullptr;
-  cudaGraphExec_t exec = nullptr;   // nullptr: capture failed, the plan runs its calls directly
-  unsigned char* dbuf = nullptr;    // [points | output]
-  size_t out_off = 0;
-  size_t scr_off = 0, scr_bytes = 0;  // the loader's SoA + box scratch inside dbuf
-  int kernels = 0;                  // kernel nodes in the graph (launch counter)
-  unsigned long long used = 0;
-  void destroy() {
-    if (exec) cudaGraphExecDestroy(exec);
-    if (dbuf) cudaFree(dbuf);
-    if (st) cudaStreamDestroy(st);
-    exec = nullptr;
-    dbuf = nullptr;
-    st = nullptr;
-  }
-};
-struct PlanCache {
-  Plan slot[kPlanSlots];
-  unsigned long long tick = 0;
-  ~PlanCache() { clear(); }
-  void clear() {
-    for (auto& p : slot) {
-      p.destroy();
-      p.key = PlanKey{};
-    }
-  }
-};
-PlanCache& plans() {
-  static thread_local PlanCache c;
-  return c;
-}
-
-// TBS_HOST_TRACE=1 (experiments): average host microseconds of the plan path's phases, printed
-// to stderr every 1000 plan calls.
-struct HostTrace {
-  bool on = getenv("TBS_HOST_TRACE") != nullptr;
-  double acc[8] = {0};
-  long calls = 0;
-  std::chrono::steady_clock::time_point t0;
-  void start() { if (on) t0 = std::chrono::steady_clock::now(); }
-  void mark(int k) {
-    if (!on) return;
-    const auto t = std::chrono::steady_clock::now();
-    acc[k] += std::chrono::duration<double, std::micro>(t - t0).count();
-    t0 = t;
-  }
-  void done() {
-    if (!on || ++calls % 1000) return;
-    fprintf(stderr, "[tbs host] per plan call (us): stage-in %.2f  H2D-enqueue %.2f  launch %.2f  D2H-enqueue %.2f  "
-            "sync %.2f  stage-out %.2f\n", acc[0] / calls, acc[1] / calls, acc[2] / calls, acc[3] / calls, acc[4] / calls,
-            acc[5] / calls);
-  }
-};
-HostTrace& host_trace() {
-  static thread_local HostTrace t;
-  return t;
-}
-
-// One host-buffer call through its plan (created, and its graph captured, on first use).
-template <class Fn>
-int run_plan(const PlanKey& key, const float* points, int pk, void* outp, int ok, size_t pbytes, size_t out_bytes,
-             Fn fn) {
-  PlanCache& pc = plans();
-  Plan* pl = nullptr;
-  for (auto& p : pc.slot)
-    if (p.key.same(key) && p.dbuf) pl = &p;
-  bool fresh = false;
-  if (!pl) {
-    pl = &pc.slot[0];
-    for (auto& p : pc.slot)
-      if (!p.dbuf || p.used < pl->used) pl = &p;     // an empty slot, else the least recently used
-    pl->destroy();
-    pl->key = key;
-    pl->out_off = (pbytes + 255) / 256 * 256;
-    pl->scr_off = (pl->out_off + out_bytes + 255) / 256 * 256;
-    pl->scr_bytes = (size_t)4 * pad_rows(key.n) * sizeof(float) + 64;   // SoA [D <= 4][n_pad] + box block
-    TBS_CUDA(cudaStreamCreateWithFlags(&pl->st, cudaStreamNonBlocking));
-    cudaError_t e = cudaMalloc((void**)&pl->dbuf, pl->scr_off + pl->scr_bytes);
-    if (e != cudaSuccess) {
-      cudaGetLastError();
-      pl->destroy();
-      pl->key = PlanKey{};
-      return fail(TBS_ENOMEM, "plan buffers (%zu B): %s", pl->scr_off + pl->scr_bytes, cudaGetErrorString(e));
-    }
-    fresh = true;
-  }
-  pl->used = ++pc.tick;
-  cudaStream_t st = pl->st;
-  tbs_args a{};
-  a.points = reinterpret_cast<const float*>(pl->dbuf);
-  a.n = key.n;
-  a.dim = key.dim;
-  a.row_begin = 0;
-  a.row_end = key.n;
-  a.stream = st;
-  void* dout = pl->dbuf + pl->out_off;
-  // pageable host buffers go through the pinned staging area: [points | output]
-  const size_t pin_in = pk == 1 ? 0 : pl->out_off, pin_out = ok == 1 ? 0 : out_bytes;
-  unsigned char* stage = nullptr;
-  if (pin_in + pin_out) {
-    void* sp = nullptr;
-    int rc = staging(pin_in + pin_out, &sp);
-    if (rc) return rc;
-    stage = static_cast<unsigned char*>(sp);
-  }
-  HostTrace& ht = host_trace();
-  ht.start();
-  const void* src = points;
-  if (pin_in) {
-    memcpy(stage, points, pbytes);
-    src = stage;
-  }
-  ht.mark(0);
-  void* dst = pin_out ? static_cast<void*>(stage + pin_in) : outp;
-  TBS_CUDA(cudaMemcpyAsync(pl->dbuf, src, pbytes, cudaMemcpyHostToDevice, st));
-  ht.mark(1);
-  int rc = TBS_OK;
-  struct ScratchScope {          // the plan's scratch for the loader while fn runs
-    explicit ScratchScope(unsigned char* p, size_t b) { plan_scratch().base = p; plan_scratch().bytes = b; }
-    ~ScratchScope() { plan_scratch() = PlanScratch{}; }
-  } scope(pl->dbuf + pl->scr_off, pl->scr_bytes);
-  if (pl->exec) {
-    TBS_CUDA(cudaGraphLaunch(pl->exec, st));
-    g_launches.fetch_add((unsigned long long)pl->kernels);
-  } else {
-    rc = fn(&a, dout);            // first call of this plan (or capture unavailable): direct launches
-  }
-  ht.mark(2);
-  if (!rc) TBS_CUDA(cudaMemcpyAsync(dst, dout, out_bytes, cudaMemcpyDeviceToHost, st));
-  ht.mark(3);
-  TBS_CUDA(cudaStreamSynchronize(st));
-  ht.mark(4);
-  if (rc) return rc;
-  if (pin_out) memcpy(outp, dst, out_bytes);
-  ht.mark(5);
-  if (!fresh) ht.done();
-  if (fresh) {
-    // capture the device work for the next calls (caches warmed by the call above); any failure
-    // leaves the plan on direct launches
-    cudaGraph_t g = nullptr;
-    if (cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal) == cudaSuccess) {
-      const int crc = fn(&a, dout);
-      const cudaError_t ce = cudaStreamEndCapture(st, &g);
-      if (crc == TBS_OK && ce == cudaSuccess && g) {
-        size_t nn = 0;
-        if (cudaGraphGetNodes(g, nullptr, &nn) == cudaSuccess && nn) {
-          std::vector<cudaGraphNode_t> nodes(nn);
-          cudaGraphGetNodes(g, nodes.data(), &nn);
-          for (auto nd : nodes) {
-            cudaGraphNodeType ty;
-            if (cudaGraphNodeGetType(nd, &ty) == cudaSuccess && ty == cudaGraphNodeTypeKernel) ++pl->kernels;
-          }
-        }
-        if (cudaGraphInstantiate(&pl->exec, g, 0) != cudaSuccess) pl->exec = nullptr;
-        g_launches.fetch_sub((unsigned long long)pl->kernels);   // captured, not launched
-      }
-      if (g) cudaGraphDestroy(g);
-    }
-    cudaGetLastError();   // a failed capture is not an error of this call
-    g_err.clear();
-  }
-  return TBS_OK;
-}
-
 // Run `fn(args_with_device_ptrs, dev_out)` for host or device buffers, synchronously.
 template <class Fn>
 int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_bytes, Fn fn,
-               PlanKey key = PlanKey{}) {
+               bool small_op = false) {
   if (n < 0 || n > TBS_MAX_N) return fail(TBS_EINVAL, "n out of range");
   if (dim < 1 || dim > 4) return fail(TBS_EINVAL, "dim out of range");
   if (!outp) return fail(TBS_EINVAL, "output is NULL");
@@ -1248,11 +1064,81 @@ int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_b
     return rc;
   }
   const size_t pbytes = (size_t)n * dim * sizeof(float);
-  if (key.op >= 0 && n >= 2 && n <= kPlanMaxN && out_bytes <= (1u << 20)) {
-    if (cudaGetDevice(&key.dev) != cudaSuccess) return fail(TBS_ECUDA, "cudaGetDevice failed");
-    key.n = n;
-    key.dim = dim;
-    return run_plan(key, points, pk, outp, ok, pbytes, out_bytes, fn);
+  if (small_op && n >= 2 && n <= kSmallLoad && out_bytes <= 65536 && out_bytes % 8 == 0) {
+    // Small problem: the copy engines' two transfers cost more than the ~10 us kernel. The
+    // points are pulled from pinned host memory (the caller's, or the staging area) by a copy
+    // kernel and the result is pushed back the same way: every step is a kernel on one stream.
+    // staging: [points (pageable input) | output (pageable output) | completion flag]
+    const size_t pin_in = pk == 1 ? 0 : (pbytes + 255) / 256 * 256;
+    const size_t pin_out = ok == 1 ? 0 : (out_bytes + 255) / 256 * 256;
+    unsigned char* stage = nullptr;
+    {
+      void* sp = nullptr;
+      if ((rc = staging(pin_in + pin_out + 64, &sp))) return rc;
+      stage = static_cast<unsigned char*>(sp);
+    }
+    volatile unsigned int* flag = reinterpret_cast<volatile unsigned int*>(stage + pin_in + pin_out);
+    void* dflag = nullptr;
+    const void* src = points;
+    if (pin_in) {
+      memcpy(stage, points, pbytes);
+      src = stage;
+    }
+    void* dst = pin_out ? static_cast<void*>(stage + pin_in) : outp;
+    void *dsrc = nullptr, *ddst = nullptr;
+    if (cudaHostGetDevicePointer(&dsrc, const_cast<void*>(src), 0) == cudaSuccess &&
+        cudaHostGetDevicePointer(&ddst, dst, 0) == cudaSuccess &&
+        cudaHostGetDevicePointer(&dflag, const_cast<unsigned int*>(flag), 0) == cudaSuccess) {
+      const size_t dp_bytes = (pbytes + 255) / 256 * 256;
+      unsigned char* dbuf = nullptr;
+      cudaError_t e = cudaMallocAsync((void**)&dbuf, dp_bytes + out_bytes + 8, st);
+      if (e != cudaSuccess) return fail(TBS_ENOMEM, "cudaMallocAsync(%zu): %s", dp_bytes + out_bytes, cudaGetErrorString(e));
+      // [points | output | ticket]; the copy kernel also zeroes output + ticket, and the fused
+      // kernel's last CTA writes the result to the mapped host buffer (else a copy kernel does)
+      const int in_words = (int)(pbytes / 4), out_words = (int)(out_bytes / 4);
+      unsigned char* dout = dbuf + dp_bytes;
+      copy_in_zero<<<(in_words + 1023) / 1024 < 8 ? (in_words + 1023) / 1024 : 8, 1024, 0, st>>>(
+          reinterpret_cast<uint32_t*>(dbuf), static_cast<const uint32_t*>(dsrc), in_words,
+          reinterpret_cast<uint32_t*>(dout), out_words + 2);
+      g_launches.fetch_add(1);
+      a.points = reinterpret_cast<const float*>(dbuf);
+      SmallWriteBack& sw = small_wb();
+      sw.wb.dst = static_cast<unsigned long long*>(ddst);
+      sw.wb.src = reinterpret_cast<const unsigned long long*>(dout);
+      sw.wb.ticket = reinterpret_cast<unsigned int*>(dout + out_bytes);
+      sw.wb.words = (int)(out_bytes / 8);
+      static thread_local unsigned int seq = 0;
+      seq = seq + 1 == 0 ? 1 : seq + 1;
+      *flag = 0u;
+      sw.wb.flag = static_cast<unsigned int*>(dflag);
+      sw.wb.seq = seq;
+      sw.active = true;
+      sw.taken = false;
+      rc = fn(&a, dout);
+      const bool taken = sw.taken;
+      sw = SmallWriteBack{};
+      if (!rc && !taken) {
+        copy_words<<<1, 256, 0, st>>>(static_cast<uint32_t*>(ddst), reinterpret_cast<const uint32_t*>(dout), out_words);
+        g_launches.fetch_add(1);
+      }
+      cudaFreeAsync(dbuf, st);
+      bool done = false;
+      if (!rc && taken) {
+        // the kernel's last CTA signals completion through the mapped flag: poll it (a stream
+        // synchronisation costs a host wake-up); give up to the synchronisation after ~50 ms
+        const auto t0 = std::chrono::steady_clock::now();
+        while (!(done = *flag == seq)) {
+          if (std::chrono::steady_clock::now() - t0 > std::chrono::milliseconds(50)) break;
+        }
+      }
+      if (!done) {
+        e = cudaStreamSynchronize(st);
+        if (!rc && e != cudaSuccess) rc = fail(TBS_ECUDA, "sync: %s", cudaGetErrorString(e));
+      }
+      if (!rc && pin_out) memcpy(outp, dst, out_bytes);
+      return rc;
+    }
+    cudaGetLastError();   // not mapped: the copy-engine path below
   }
   // pageable buffers go through the pinned staging area: [points | output]
   size_t pin_in = pk == 1 ? 0 : (pbytes + 255) / 256 * 256;
@@ -1313,22 +1199,15 @@ int tbs_pairmatrix_ex(const tbs_args* args, tbs_kernel kernel, float* out) {
 int tbs_sdh(const float* points, int64_t n, int dim, float bucket_width, int nbuckets, uint64_t* hist) {
   g_err.clear();
   if (nbuckets < 1 || nbuckets > TBS_MAX_BUCKETS) return fail(TBS_EINVAL, "nbuckets out of range");
-  PlanKey key;
-  key.op = 0;
-  key.f = bucket_width;
-  key.i = nbuckets;
   return run_simple(points, n, dim, hist, (size_t)nbuckets * 8, [&](tbs_args* a, void* out) {
     return sdh_impl(a, bucket_width, nbuckets, (uint64_t*)out);
-  }, key);
+  }, true);
 }
 
 int tbs_pcf(const float* points, int64_t n, float radius, uint64_t* count) {
   g_err.clear();
-  PlanKey key;
-  key.op = 1;
-  key.f = radius;
   return run_simple(points, n, 3, count, 8, [&](tbs_args* a, void* out) { return pcf_impl(a, radius, (uint64_t*)out); },
-                    key);
+                    true);
 }
 
 int tbs_pairmatrix(const float* points, int64_t n, tbs_kernel kernel, float* out) {
@@ -1345,10 +1224,7 @@ int tbs_kde_ex(const tbs_args* args, float gamma, double* sum) {
 
 int tbs_kde(const float* points, int64_t n, float gamma, double* sum) {
   g_err.clear();
-  PlanKey key;
-  key.op = 2;
-  key.f = gamma;
-  return run_simple(points, n, 3, sum, 8, [&](tbs_args* a, void* out) { return kde_impl(a, gamma, (double*)out); }, key);
+  return run_simple(points, n, 3, sum, 8, [&](tbs_args* a, void* out) { return kde_impl(a, gamma, (double*)out); }, true);
 }
 
 int tbs_rdf_ex(const tbs_args* args, float bucket_width, int nbuckets, double volume, double* g) {
@@ -1530,7 +1406,6 @@ int tbs_peer_atomics_ok(const char* pci_bus_id, int* ok) {
 const char* tbs_last_error(void) { return g_err.c_str(); }
 
 void tbs_release(void) {
-  plans().clear();
   int dev;
   if (cudaGetDevice(&dev) != cudaSuccess) return;
   cudaMemPool_t pool;

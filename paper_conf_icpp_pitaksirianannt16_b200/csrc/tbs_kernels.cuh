@@ -915,9 +915,23 @@ __global__ void push_peers(const unsigned long long* __restrict__ acc, int words
 // SoA layout run_chunk reads), so the call is one memset of the output plus this launch
 // instead of a loader launch plus the pair kernel (the loader was ~7 us of a ~20 us step).
 // No bounding box exists here: float SDH takes the clamp variant V.
+// WriteBack (host-buffer calls): the last CTA to finish copies the `words` u64 of the result
+// at `src` to mapped page-locked host memory `dst` (ticket zeroed before the launch).
+// Then it stores `seq` to the mapped host word `flag` (after a system fence), which the host
+// polls instead of waiting in a stream synchronisation.
+struct WriteBack {
+  unsigned long long* dst = nullptr;
+  const unsigned long long* src = nullptr;
+  unsigned int* ticket = nullptr;
+  int words = 0;
+  unsigned int* flag = nullptr;
+  unsigned int seq = 0;
+};
+
 template <class Op, int D, class C, int V>
 __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel_small(const float* __restrict__ pts, int dim, Geom g,
-                                                                  Op op, const __grid_constant__ OutSink sink) {
+                                                                  Op op, const __grid_constant__ OutSink sink,
+                                                                  const WriteBack wb) {
   unsigned char* smem = tbs_smem;
   const long long hbytes = (op.smem_bytes() + 127) & ~127ll;
   float* B = reinterpret_cast<float*>(smem + hbytes);
@@ -949,6 +963,38 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel_small(const flo
   else run_chunk<Op, D, C, true, V>(op, B, na, g, I, p0, cnt);
   __syncthreads();
   op.finish(smem);
+  if (wb.dst != nullptr) {
+    __shared__ unsigned int s_last;
+    __threadfence();                       // this CTA's output atomics before its ticket
+    __syncthreads();
+    if (tid == 0) s_last = atomicAdd(wb.ticket, 1u) == gridDim.x - 1 ? 1u : 0u;
+    __syncthreads();
+    if (s_last) {
+      __threadfence();
+      for (int k = tid; k < wb.words; k += kThreads) wb.dst[k] = __ldcg(wb.src + k);
+      __threadfence_system();
+      __syncthreads();
+      if (tid == 0 && wb.flag != nullptr) {
+        *reinterpret_cast<volatile unsigned int*>(wb.flag) = wb.seq;
+        __threadfence_system();
+      }
+    }
+  }
+}
+
+// Host-buffer small calls: copy the points from mapped page-locked host memory and zero the
+// output words (+ the write-back ticket) the fused kernel accumulates into.
+__global__ void copy_in_zero(uint32_t* __restrict__ dst, const uint32_t* __restrict__ src, int words,
+                             uint32_t* __restrict__ zero, int zero_words) {
+  const int stride = gridDim.x * blockDim.x;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < words; i += stride) dst[i] = src[i];
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < zero_words; i += stride) zero[i] = 0u;
+}
+
+// Word copy between device memory and mapped (page-locked) host memory: the small-problem
+// host-buffer path moves its few kilobytes with kernels instead of copy-engine transfers.
+__global__ void copy_words(uint32_t* __restrict__ dst, const uint32_t* __restrict__ src, int words) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < words; i += gridDim.x * blockDim.x) dst[i] = src[i];
 }
 
 // Sum G partial global copies into the output (one thread per bin, the paper's

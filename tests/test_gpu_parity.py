@@ -627,23 +627,23 @@ def test_validate_flag(tbs):
     torch.cuda.synchronize()
 
 
-# ------------------------------------------------------------------ small-problem plans (graph-captured host calls)
-def test_host_plan_cache(tbs):
-    """Host-buffer calls with n <= 64K go through per-thread plans (a CUDA graph captured on the
-    first call of a key): repeated calls, interleaved keys, more keys than plan slots (LRU
-    eviction), pageable and pinned buffers and tbs_release() all give the oracle's result."""
+# ------------------------------------------------------------------ small-problem host-buffer path
+def test_host_small_path(tbs):
+    """Host-buffer calls with n <= 16K move points and result with copy kernels over mapped
+    pinned memory (the caller's pinned buffers, or the staging area for pageable ones) around
+    the fused small-problem kernel: repeated and interleaved calls, pageable and pinned buffers,
+    many radii, and the sizes around the switch all give the oracle's result."""
     import torch
     nb = 64
-    pts = {n: g.uniform(n, 300 + n) for n in (2, 3000, 4096, 65536)}
-    want = {n: oracle.sdh(p, w_of(nb), nb) for n, p in pts.items() if n <= 4096}
+    pts = {n: g.uniform(n, 300 + n) for n in (2, 3000, 4096, 16384, 65536)}
+    want = {n: oracle.sdh(p, w_of(nb), nb) for n, p in pts.items() if n <= 16384}
     for rep in range(3):
-        for n in (2, 3000, 4096):
+        for n in (2, 3000, 4096, 16384):
             h = tbs.sdh_host(pts[n], w_of(nb), nb)
             check_sdh_float(h, *want[n])
     pin = torch.from_numpy(pts[4096]).pin_memory()
     for _ in range(3):
         check_sdh_float(tbs.sdh_host(pin.numpy(), w_of(nb), nb), *want[4096])
-    # 10 distinct keys (> 8 slots): eviction, then the first keys again
     for k in list(range(10)) + [0, 1]:
         r = 0.02 + 0.01 * k
         c = tbs.pcf_host(pts[3000], r)
@@ -651,6 +651,6 @@ def test_host_plan_cache(tbs):
         check_pcf_float(c, co, ca)
     tbs.release()
     check_sdh_float(tbs.sdh_host(pts[3000], w_of(nb), nb), *want[3000])
-    h = tbs.sdh_host(pts[65536], w_of(nb), nb)                     # the largest planned n
+    h = tbs.sdh_host(pts[65536], w_of(nb), nb)                     # above the small-problem switch
     assert int(h.sum()) == 65536 * 65535 // 2
     assert h.tolist() == tbs.sdh(dev(pts[65536]), w_of(nb), nb).cpu().tolist()
