@@ -73,6 +73,49 @@ def make(name, part=None, parts=None, outdir=None):
     print(fn, out["oracle_seconds"], "s")
 
 
+def make_split(name, part, parts, outdir, split):
+    """Part `part` of `parts` computed as `split` pair-balanced anchor-row sub-ranges, one
+    oracle call each (every call uses all OpenMP threads on rows of similar cost: a single call
+    over a long triangular range leaves the threads holding its first, heaviest guided chunks
+    running long after the others). The sub-range outputs are integer counts and add up to
+    the part's; the file is the same as make(name, part, parts) writes."""
+    spec = GOLDENS[name]
+    n = spec["n"]
+    p = g.make(spec["kind"], n, spec["seed"])
+    b, e = part_rows(n, parts, part)
+    # sub-range boundaries with equal pair counts inside [b, e)
+    S = lambda x: x * (2 * n - x - 1) // 2
+    tot = S(e) - S(b)
+    bounds = [b]
+    for k in range(1, split):
+        target = S(b) + tot * k // split
+        lo, hi = bounds[-1], e
+        while lo < hi:
+            mid = (lo + hi) // 2
+            if S(mid) < target:
+                lo = mid + 1
+            else:
+                hi = mid
+        bounds.append(lo)
+    bounds.append(e)
+    t0 = time.time()
+    w = float(np.float32(math.sqrt(3) / spec["nb"]))
+    hist = np.zeros(spec["nb"], np.uint64)
+    amb = np.zeros(spec["nb"] + 1, np.uint64)
+    for k in range(split):
+        h, a = oracle.sdh(p, w, spec["nb"], rows=(bounds[k], bounds[k + 1]))
+        hist += h
+        amb += a
+        print(f"sub-range {k + 1}/{split} rows [{bounds[k]}, {bounds[k + 1]}) {time.time() - t0:.0f} s", flush=True)
+    out = dict(name=name, spec=spec, generator="tbs_inputs." + spec["kind"], script="tools/make_goldens.py",
+               threads=oracle.num_threads(), rows=[b, e], part=part, parts=parts, split=split,
+               w=w, hist=[int(x) for x in hist], amb=[int(x) for x in amb], oracle_seconds=round(time.time() - t0, 2))
+    fn = f"{name}.part{part}of{parts}.json"
+    with open(os.path.join(outdir, fn), "w") as f:
+        json.dump(out, f, indent=0)
+    print(fn, out["oracle_seconds"], "s")
+
+
 def merge(name, files):
     """Sum the parts' oracle outputs (integer counts: order-independent) into the golden."""
     ds = [json.load(open(f)) for f in files]
@@ -94,10 +137,13 @@ def merge(name, files):
 if __name__ == "__main__":
     # python tools/make_goldens.py NAME...                    full goldens
     # python tools/make_goldens.py --part K PARTS OUTDIR NAME  one pair-balanced row part
+    # python tools/make_goldens.py --part-split K PARTS OUTDIR NAME SPLIT   the part as SPLIT sub-ranges
     # python tools/make_goldens.py --merge NAME PART_FILE...   sum the parts
     a = sys.argv[1:]
     if a and a[0] == "--part":
         make(a[4], int(a[1]), int(a[2]), a[3])
+    elif a and a[0] == "--part-split":      # --part-split K PARTS OUTDIR NAME SPLIT (SDH goldens)
+        make_split(a[4], int(a[1]), int(a[2]), a[3], int(a[5]))
     elif a and a[0] == "--merge":
         merge(a[1], a[2:])
     else:
