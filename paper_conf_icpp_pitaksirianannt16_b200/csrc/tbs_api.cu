@@ -1027,7 +1027,7 @@ int staging(size_t bytes, void** out) {
     s.p = nullptr;
     s.bytes = 0;
     const size_t want = std::max<size_t>(bytes, 1 << 20);
-    if (cudaHostAlloc(&s.p, want, cudaHostAllocDefault) != cudaSuccess) {
+    if (cudaHostAlloc(&s.p, want, cudaHostAllocPortable | cudaHostAllocMapped) != cudaSuccess) {
       cudaGetLastError();
       return fail(TBS_ENOMEM, "cudaHostAlloc(%zu) for host staging failed", want);
     }

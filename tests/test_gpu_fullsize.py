@@ -316,3 +316,28 @@ def test_knn_lattice_2_5m_exact_strips(tbs):
     for rb, re in strips(n, 8):
         oi, od = oracle.knn(p, k, rows=(rb, re))
         assert np.array_equal(gi[rb:re], oi) and np.array_equal(gd[rb:re], od.astype(np.float32))
+
+
+# ---------------------------------------------------------------- maximum size (TBS_MAX_N = 2^30)
+def test_max_n_strips(tbs):
+    """n = TBS_MAX_N = 2^30 (12 GiB of points, 12 GiB of SoA scratch): every index the kernels
+    form (tiles, chunks, SoA offsets, row bounds) stays in range. Points are coincident except
+    the last, at distance 5 (w = 1, exact), so each strip's histogram is known in closed form:
+    anchor i pairs with n-1-i partners, all at distance 0 except the pair with the last point."""
+    import torch
+    n = 1 << 30
+    p = torch.zeros((n, 3), dtype=torch.float32, device="cuda")
+    p[n - 1, 0] = 3.0
+    p[n - 1, 1] = 4.0
+    try:
+        for rows in ((0, 1), (n - 5000, n - 2000), (n - 2, n)):
+            b, e = rows
+            h = tbs.sdh(p, 1.0, 8, rows=rows, lattice=True).cpu().numpy()
+            pairs = (e - b) * (2 * n - b - e - 1) // 2
+            far = e - b if e < n else e - b - 1          # pairs (i, n-1) with i in the strip, i < n-1
+            assert int(h.sum()) == pairs and int(h[5]) == far and int(h[0]) == pairs - far, (rows, h)
+            c = int(tbs.pcf(p, 4.5, rows=rows).item())
+            assert c == pairs - far
+    finally:
+        del p
+        torch.cuda.empty_cache()

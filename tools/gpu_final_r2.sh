@@ -29,4 +29,6 @@ for tool in memcheck racecheck synccheck initcheck; do
   echo "$tool exit $?"
 done
 timeout 300 python tools/c1_e2e.py > $O/c1_e2e.json 2>&1
+timeout 900 python tools/partition_balance.py > $O/partition_balance.jsonl 2>&1
+timeout 900 python tools/ablations.py > $O/ablations.jsonl 2>&1
 ls -la $O
