@@ -141,11 +141,13 @@ def test_sdh_4m_uniform_strips_and_mass(tbs):
         check_sdh_float(hs, ho, amb)
 
 
-def test_sdh_4m_uniform_vs_golden_part(tbs):
-    """North-star workload at full size on its first pair-balanced anchor-row part (rows
-    [0, 1228483): half of the 8.8e12 pairs), against the CPU oracle's histogram of exactly
-    those pairs (tools/make_goldens.py --part 0 2, 43 min on 16 host threads)."""
-    gold = json.load(open(os.path.join(GOLD, "parts", "sdh_uniform_n4194304_nb256_seed6.part0of2.json")))
+@pytest.mark.parametrize("part", [0, 1])
+def test_sdh_4m_uniform_vs_golden_part(tbs, part):
+    """North-star workload at full size on each pair-balanced anchor-row part (rows [0, 1228483)
+    and [1228483, 4194304): half of the 8.8e12 pairs each) through the row-range API, against the
+    CPU oracle's histogram of exactly those pairs (tools/make_goldens.py --part 0 2: 43 min;
+    --part-split 1 2 ... 48: 43 min, both on a GPU box's 16 host threads)."""
+    gold = json.load(open(os.path.join(GOLD, "parts", f"sdh_uniform_n4194304_nb256_seed6.part{part}of2.json")))
     n = gold["spec"]["n"]
     rb, re = gold["rows"]
     p = g.uniform(n, gold["spec"]["seed"])
@@ -153,16 +155,14 @@ def test_sdh_4m_uniform_vs_golden_part(tbs):
     d = check_sdh_float(h, gold["hist"], gold["amb"])
     # pairs (i, j), rb <= i < re, i < j < n
     assert int(h.sum()) == sum(gold["hist"]) == (re - rb) * (2 * n - rb - re - 1) // 2
-    print("4M golden part 0:", d)
+    print(f"4M golden part {part}:", d)
 
 
 def test_sdh_4m_uniform_vs_golden(tbs):
     """North-star workload at full size, whole histogram (bench.py's default launch, all
     8.8e12 pairs) against the merged oracle golden (both pair-balanced parts)."""
-    gp = os.path.join(GOLD, "sdh_uniform_n4194304_nb256_seed6.json")
-    if not os.path.exists(gp):
-        pytest.skip("part 1 of the 4M SDH golden not yet computed (DESIGN §3)")
-    gold = json.load(open(gp))
+    gold = json.load(open(os.path.join(GOLD, "sdh_uniform_n4194304_nb256_seed6.json")))
+    assert gold["merged_parts"] == [[0, 1228483], [1228483, 4194304]]
     n = gold["spec"]["n"]
     p = g.uniform(n, gold["spec"]["seed"])
     h = host(tbs.sdh(dev(p), gold["w"], 256)).astype(np.uint64)

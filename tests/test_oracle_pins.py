@@ -459,3 +459,23 @@ def test_knn_k_exceeds_n_minus_1_and_rows():
     full_i, full_d = oracle.knn(q, 4)
     part_i, part_d = oracle.knn(q, 4, rows=(100, 170))
     assert np.array_equal(part_i, full_i[100:170]) and np.array_equal(part_d, full_d[100:170])
+
+
+def test_4m_golden_parts_merge():
+    """The north-star golden (tools/make_goldens.py, oracle only) is the sum of its two
+    pair-balanced parts; each part's mass is the pair count of its anchor rows and the whole
+    is C(n, 2); every ambiguity count is bounded by its neighbouring buckets' mass."""
+    base = os.path.join(GOLDEN, "sdh_uniform_n4194304_nb256_seed6")
+    full = json.load(open(base + ".json"))
+    parts = [json.load(open(os.path.join(GOLDEN, "parts", f"sdh_uniform_n4194304_nb256_seed6.part{k}of2.json")))
+             for k in (0, 1)]
+    n = full["spec"]["n"]
+    assert sum(full["hist"]) == n * (n - 1) // 2
+    for pt in parts:
+        b, e = pt["rows"]
+        assert sum(pt["hist"]) == (e - b) * (2 * n - b - e - 1) // 2
+        assert pt["w"] == full["w"] == float(np.float32(math.sqrt(3) / 256))
+    assert [x + y for x, y in zip(parts[0]["hist"], parts[1]["hist"])] == full["hist"]
+    assert [x + y for x, y in zip(parts[0]["amb"], parts[1]["amb"])] == full["amb"]
+    h, a = full["hist"], full["amb"]
+    assert all(a[k] <= h[k - 1] + h[k] for k in range(1, 256))
