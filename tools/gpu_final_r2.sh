@@ -17,11 +17,16 @@ for wl in sdh_uniform_4m sdh_clustered_1m sdh_uniform_2m_16k sdh_lattice_4m sdh_
 done
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_sdh_uniform_1m.csv \
   python bench.py --steps 2 --warmup 3 --no-cpu-baseline > $O/launches.log 2>&1
+# ncu reports stay on the box (gpurun copies back <= 64 MiB): keep their summaries and details
 for wl in sdh_uniform_1m sdh_uniform_2m_16k pcf_clustered_4m; do
-  ncu --set full --clock-control none --import-source on -k regex:pair_kernel -s 3 -c 1 -o $O/prof_$wl \
+  ncu --set full --clock-control none --import-source on -k regex:pair_kernel -s 3 -c 1 -o /tmp/prof_$wl \
     python bench.py --workload $wl --steps 1 --warmup 3 --no-cpu-baseline > $O/ncu_$wl.log 2>&1
+  python tools/ncu_summary.py /tmp/prof_$wl.ncu-rep > $O/ncu_summary_$wl.txt 2>&1
+  ncu -i /tmp/prof_$wl.ncu-rep --page details > $O/ncu_details_$wl.txt 2>&1
 done
-ncu --set full --clock-control none --import-source on -k regex:"pair_kernel|soa_loader" -s 40 -c 2 -o $O/prof_c1 python tools/c1_probe.py > $O/ncu_c1.log 2>&1
+ncu --set full --clock-control none --import-source on -k regex:"pair_kernel" -s 20 -c 1 -o /tmp/prof_c1 python tools/c1_probe.py > $O/ncu_c1.log 2>&1
+python tools/ncu_summary.py /tmp/prof_c1.ncu-rep > $O/ncu_summary_c1.txt 2>&1
+du -sh $O
 ./tools/peaks > $O/peaks.json 2>&1
 nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o /tmp/ablate_intra tools/ablate_intra.cu && /tmp/ablate_intra > $O/ablate_intra.jsonl 2>&1
 for tool in memcheck racecheck synccheck initcheck; do
