@@ -152,3 +152,56 @@ def test_fused_two_processes_ipc(tbs):
     assert res[0][2:4] == res[1][2:4]
     for pr in procs:
         assert pr.exitcode == 0
+
+
+def _nccl_worker(port, q):
+    """A one-rank NCCL group on the GPU: the binding's group path (pair-balanced strip of a
+    world-1 partition = all rows, then tbs.combine's all_reduce over NCCL on a device tensor)."""
+    import torch
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    torch.cuda.set_device(0)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda:0"))
+    try:
+        import paper_conf_icpp_pitaksirianannt16_b200 as tbs
+        G = dist.group.WORLD
+        pl = torch.from_numpy(g.lattice(20, 37)).cuda()
+        pc = torch.from_numpy(g.clustered(30000, 38)).cuda()
+        w = float(np.float32(math.sqrt(3) / 128))
+        out = {
+            "backend": dist.get_backend(G),
+            "hl": tbs.sdh(pl, 0.5, 70, lattice=True, group=G).cpu().tolist(),
+            "hf": tbs.sdh(pc, w, 128, group=G).cpu().tolist(),
+            "hf1": tbs.sdh(pc, w, 128).cpu().tolist(),
+            "c": int(tbs.pcf(pc, 0.03, group=G).cpu()[0]),
+            "c1": int(tbs.pcf(pc, 0.03).cpu()[0]),
+            "kde": float(tbs.kde(pc[:5000], 2.0, group=G).cpu()[0]),
+            "kde1": float(tbs.kde(pc[:5000], 2.0).cpu()[0]),
+        }
+        q.put(out)
+    except Exception as e:
+        q.put({"error": repr(e)})
+        raise
+    finally:
+        dist.destroy_process_group()
+
+
+def test_nccl_combine_world1():
+    """The north star's combine (one NCCL all_reduce of the rank partials) executed on the GPU:
+    one rank, so the result must equal the ungrouped call bit for bit and the oracle's rule."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    pr = ctx.Process(target=_nccl_worker, args=(_free_port(), q))
+    pr.start()
+    r = q.get(timeout=600)
+    pr.join(timeout=120)
+    assert "error" not in r, r
+    assert r["backend"] == "nccl"
+    assert r["hl"] == oracle.sdh_lattice(g.lattice(20, 37), 1, 1, 70).astype(np.int64).tolist()
+    assert r["hf"] == r["hf1"] and r["c"] == r["c1"]
+    assert abs(r["kde"] - r["kde1"]) <= 1e-12 * abs(r["kde1"])   # fp64 partial sums: order may vary
+    pc = g.clustered(30000, 38)
+    cw, camb = oracle.pcf(pc, 0.03)
+    assert abs(r["c"] - int(cw)) <= int(camb)
+    assert pr.exitcode == 0
