@@ -28,6 +28,20 @@ static_assert(kMaxPeers == TBS_MAX_PEERS, "peer sink size");
 
 // Pair-engine configurations per output type: anchors/thread, partner chunk, CTAs/SM
 // (A/B-tunable with -D at build time, see tools/build_ab.py).
+// tensor-core pair matrix (tbs_hd2.cuh): operand ring stages / epilogue staging buffers for
+// small d (<= 128: at most 2 k-blocks per tile) and large d
+#ifndef TBS_HD2_RING_S
+#define TBS_HD2_RING_S 4
+#endif
+#ifndef TBS_HD2_NSTG_S
+#define TBS_HD2_NSTG_S 2
+#endif
+#ifndef TBS_HD2_RING_L
+#define TBS_HD2_RING_L 4
+#endif
+#ifndef TBS_HD2_NSTG_L
+#define TBS_HD2_NSTG_L 2
+#endif
 #ifndef TBS_SDH_KA
 #define TBS_SDH_KA 8
 #endif
@@ -881,7 +895,12 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
                             : 2 * (int)std::min<long long>(ntiles, dev.sms / 2);   // CTA pairs
     const float cexp = (float)(-(double)k.gamma * 1.4426950408889634);
     const int kblocks = dp / hd::kKBlock;
-    const int smem = (one_sm ? hd::Smem::BYTES : hd2::Smem::BYTES) + 1024;
+    // CTA-pair kernel shape (operand ring depth, epilogue staging buffers): small d (<= 2
+    // k-blocks per tile, output-bound) vs large d.
+    const bool small_d = kblocks <= 2;
+    using SmemS = hd2::Smem<TBS_HD2_RING_S, TBS_HD2_NSTG_S>;
+    using SmemL = hd2::Smem<TBS_HD2_RING_L, TBS_HD2_NSTG_L>;
+    const int smem = (one_sm ? hd::Smem::BYTES : small_d ? SmemS::BYTES : SmemL::BYTES) + 1024;
     // CTA-pair tile raster: bands of `band` tile rows walked column by column, tiles dealt
     // round-robin over clusters (0: contiguous row-major range per cluster). TBS_HD_BAND overrides.
     static const int band_env = [] { const char* e = getenv("TBS_HD_BAND"); return e ? atoi(e) : -1; }();
@@ -894,7 +913,7 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
     auto launch = [&](auto kern) -> int {
       TBS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
       if (eb) TBS_CUDA(cudaEventRecord(eb, st));
-      if constexpr (std::is_same<decltype(kern), decltype(&hd2::hd_pair_kernel<0>)>::value)
+      if constexpr (std::is_same<decltype(kern), decltype(&hd2::hd_pair_kernel<0, 4, 2>)>::value)
         kern<<<grid, hd2::kThreads, smem, st>>>(tmap, tmap_out, use_tma_store, norms, (int)n, kblocks, I0, tiles_i,
                                                 tiles_j, (int)rb, (int)re, cexp, out, band);
       else
@@ -909,10 +928,14 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
       rc = k.type == 0 ? launch(hd::hd_pairmatrix_kernel<0>)
            : k.type == 1 ? launch(hd::hd_pairmatrix_kernel<1>)
                          : launch(hd::hd_pairmatrix_kernel<2>);
+    else if (small_d)
+      rc = k.type == 0 ? launch(hd2::hd_pair_kernel<0, TBS_HD2_RING_S, TBS_HD2_NSTG_S>)
+           : k.type == 1 ? launch(hd2::hd_pair_kernel<1, TBS_HD2_RING_S, TBS_HD2_NSTG_S>)
+                         : launch(hd2::hd_pair_kernel<2, TBS_HD2_RING_S, TBS_HD2_NSTG_S>);
     else
-      rc = k.type == 0 ? launch(hd2::hd_pair_kernel<0>)
-           : k.type == 1 ? launch(hd2::hd_pair_kernel<1>)
-                         : launch(hd2::hd_pair_kernel<2>);
+      rc = k.type == 0 ? launch(hd2::hd_pair_kernel<0, TBS_HD2_RING_L, TBS_HD2_NSTG_L>)
+           : k.type == 1 ? launch(hd2::hd_pair_kernel<1, TBS_HD2_RING_L, TBS_HD2_NSTG_L>)
+                         : launch(hd2::hd_pair_kernel<2, TBS_HD2_RING_L, TBS_HD2_NSTG_L>);
   }
   cudaFreeAsync(scratch, st);
   return rc;

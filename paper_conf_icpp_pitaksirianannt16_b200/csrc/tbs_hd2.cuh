@@ -14,7 +14,7 @@
 //   * commits are multicast to both CTAs (operand stage free, accumulator full); both
 //     CTAs' epilogues release the accumulator on the leader's barrier;
 //   * each CTA's 16 epilogue warps drain its 128 x 256 accumulator in four 64-column quarters
-//     through two 32 KB swizzled staging buffers (double-buffered) and 2-D TMA stores.
+//     through NSTG 32 KB swizzled staging buffers (in turn) and 2-D TMA stores.
 #pragma once
 #include <cstdint>
 #include "tbs_hd.cuh"
@@ -28,7 +28,10 @@ using hd::kKBlock;
 using hd::kStageBytes;
 constexpr int kPair = 256;                         // output tile of a CTA pair (M = N = 256)
 constexpr int kHalf = 128;                         // rows (and B rows) per CTA
-constexpr int kRing = 4;                           // operand ring: 4 x (A 16 KB | B 16 KB) per CTA
+// Operand ring depth and epilogue staging buffers are template parameters (RING x 32 KB of
+// operands + NSTG x 32 KB of staging fit 227 KB for RING + NSTG <= 6): deep rings for large d
+// (many k-blocks per tile), more staging buffers — more TMA store groups in flight — when the
+// output stream is the bound (small d).
 constexpr int kThreads = (kEpiWarps + 2) * 32;     // + a TMA producer warp and an MMA warp
 constexpr int kTmemCols = 512;                     // two 256-column fp32 accumulators
 constexpr int kNorms = kHalf + kPair;              // per slot: 128 row norms | 256 column norms
@@ -36,14 +39,15 @@ constexpr uint32_t kPeerMask = 0xFEFFFFFFu;        // clears the CTA-rank bit of
 constexpr int kQuarter = 64;                       // columns per epilogue staging step
 constexpr int kStageBuf = kHalf * kQuarter * 4;    // 32 KB per staging buffer
 
+template <int RING, int NSTG>
 struct Smem {
-  static constexpr int OPS = 0;                              // [kRing][A | B] x 16 KB
+  static constexpr int OPS = 0;                              // [RING][A | B] x 16 KB
   static constexpr int OPS_STAGE = 2 * kStageBytes;
-  static constexpr int STAGE = OPS + kRing * OPS_STAGE;      // 2 x (128 x 64 fp32) staging (2 swizzled boxes each)
-  static constexpr int NORMS = STAGE + kHalf * kHalf * 4;    // [4 slots][kNorms] fp32
+  static constexpr int STAGE = OPS + RING * OPS_STAGE;       // NSTG x (128 x 64 fp32) staging (2 swizzled boxes each)
+  static constexpr int NORMS = STAGE + NSTG * kStageBuf;     // [4 slots][kNorms] fp32
   static constexpr int BARS = NORMS + 4 * kNorms * 4;
-  // full[kRing] free[kRing] acc_full[2] acc_empty[2] nfull[4] nempty[4]
-  static constexpr int TMEM = BARS + (2 * kRing + 12) * 8;
+  // full[RING] free[RING] acc_full[2] acc_empty[2] nfull[4] nempty[4]
+  static constexpr int TMEM = BARS + (2 * RING + 12) * 8;
   static constexpr int BYTES = TMEM + 16;
 };
 
@@ -71,7 +75,8 @@ __device__ __forceinline__ uint32_t map_rank(uint32_t a, uint32_t rank) {
 __device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
   asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
 }
-__device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
 // 32 lanes x 16 consecutive 32-bit TMEM columns -> 16 registers per thread.
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
   asm volatile(
@@ -118,24 +123,25 @@ __device__ __forceinline__ void commit_pair(uint32_t bar) {
       : "memory");
 }
 
-template <int KTYPE>
+template <int KTYPE, int RING, int NSTG>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     hd_pair_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ CUtensorMap tmap_out,
                    int use_tma_store, const float* __restrict__ norms, int n, int kblocks, int I0, int tiles_i,
                    int tiles_j, int rb, int re, float cexp, float* __restrict__ out, int band) {
+  using SM = Smem<RING, NSTG>;
   extern __shared__ __align__(1024) unsigned char hd2_smem_raw[];
   unsigned char* sm = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(hd2_smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sbase = smem_addr(sm);
-  const uint32_t b0 = sbase + Smem::BARS;
+  const uint32_t b0 = sbase + SM::BARS;
   auto bar_full = [&](int s) { return b0 + 8 * s; };
-  auto bar_free = [&](int s) { return b0 + 8 * (kRing + s); };
-  auto bar_acc_full = [&](int a) { return b0 + 8 * (2 * kRing + a); };
-  auto bar_acc_empty = [&](int a) { return b0 + 8 * (2 * kRing + 2 + a); };
-  auto bar_nfull = [&](int k) { return b0 + 8 * (2 * kRing + 4 + k); };
-  auto bar_nempty = [&](int k) { return b0 + 8 * (2 * kRing + 8 + k); };
-  const uint32_t stage = sbase + Smem::STAGE;
-  const uint32_t snorm = sbase + Smem::NORMS;
-  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(sm + Smem::TMEM);
+  auto bar_free = [&](int s) { return b0 + 8 * (RING + s); };
+  auto bar_acc_full = [&](int a) { return b0 + 8 * (2 * RING + a); };
+  auto bar_acc_empty = [&](int a) { return b0 + 8 * (2 * RING + 2 + a); };
+  auto bar_nfull = [&](int k) { return b0 + 8 * (2 * RING + 4 + k); };
+  auto bar_nempty = [&](int k) { return b0 + 8 * (2 * RING + 8 + k); };
+  const uint32_t stage = sbase + SM::STAGE;
+  const uint32_t snorm = sbase + SM::NORMS;
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(sm + SM::TMEM);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cta_rank();
   const int cid = (int)(blockIdx.x >> 1), nclusters = (int)(gridDim.x >> 1);
@@ -165,7 +171,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
 
   if (warp == kEpiWarps) {
     if (lane == 0) {
-      for (int k = 0; k < kRing; ++k) {
+      for (int k = 0; k < RING; ++k) {
         mbar_init(bar_full(k), 1);
         mbar_init(bar_free(k), 1);
       }
@@ -218,18 +224,18 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
         if (reuse) mbar_wait(bar_free(st), ph ^ 1u);     // the pair's MMAs of the previous pass done
         if (hd::elect_one()) {
           if (rank == 0) mbar_arrive_expect_tx(bar_full(st), (uint32_t)(2 * 2 * kStageBytes));   // both CTAs' bytes
-          const uint32_t ops = sbase + Smem::OPS + st * Smem::OPS_STAGE;
+          const uint32_t ops = sbase + SM::OPS + st * SM::OPS_STAGE;
           tma_load_2d_pair(ops, &tmap, kb * kKBlock, I * kPair + rank * kHalf, bar_full(st), keep);
           tma_load_2d_pair(ops + kStageBytes, &tmap, kb * kKBlock, J * kPair + rank * kHalf, bar_full(st), keep);
         }
         __syncwarp();
-        if (++st == kRing) { st = 0; ph ^= 1u; reuse = true; }
+        if (++st == RING) { st = 0; ph ^= 1u; reuse = true; }
       }
     }
   } else if (warp == kEpiWarps + 1) {
     if (rank == 0) {
       // MMA issuer of the pair (leader CTA only).
-      const uint64_t dbase = hd::sw128_desc(sbase + Smem::OPS);
+      const uint64_t dbase = hd::sw128_desc(sbase + SM::OPS);
       int st = 0;
       uint32_t ph = 0u;
       for (long long t = 0; t < my_tiles; ++t) {
@@ -239,10 +245,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
         for (int kb = 0; kb < kblocks; ++kb) {
           mbar_wait(bar_full(st), ph);
           hd::tc_fence_after();
-          const uint64_t da = dbase + (uint64_t)((st * Smem::OPS_STAGE) >> 4);
+          const uint64_t da = dbase + (uint64_t)((st * SM::OPS_STAGE) >> 4);
           if (hd::elect_one()) mma_kblock_pair(d_tmem, da, da + (uint64_t)(kStageBytes >> 4), kb != 0 ? 1u : 0u, bar_free(st));
           __syncwarp();
-          if (++st == kRing) { st = 0; ph ^= 1u; }
+          if (++st == RING) { st = 0; ph ^= 1u; }
         }
         if (hd::elect_one()) commit_pair(bar_acc_full(acc));
         __syncwarp();
@@ -250,15 +256,16 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     }
   } else {
     // Epilogue warps: TMEM lane quarter q; each 256-column accumulator row block drains in
-    // four 64-column quarters (warp column chunk cq = 16 columns of a quarter) through TWO
-    // 32 KB staging buffers: quarter k is written while the TMA stores of quarter k-1 are
-    // still reading the other buffer, so the store stream (the HBM-bound part) never waits
-    // for the compute of the next quarter.
+    // four 64-column quarters (warp column chunk cq = 16 columns of a quarter) through NSTG
+    // 32 KB staging buffers used in turn: quarter k is written while the TMA stores of the
+    // NSTG - 1 quarters before it may still be reading theirs, so the store stream (the
+    // HBM-bound part) never waits for the compute of the next quarter.
     const int q = warp & 3, cq = warp >> 2;
     const int r = 32 * q + lane;
     const uint64_t stream_out = hd::policy_evict_first();
     const bool storer = threadIdx.x == 0;
     const uint32_t acc_empty_leader[2] = {map_rank(bar_acc_empty(0), 0), map_rank(bar_acc_empty(1), 0)};
+    int qs = 0;                                            // staging buffer of the next quarter
     for (long long t = 0; t < my_tiles; ++t) {
       int I, J;
       tile_ij(t, I, J);
@@ -293,8 +300,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
           else if (KTYPE == 1) o[x] = fmaxf(s, 0.f);
           else o[x] = sqrt_approx(fmaxf(s, 0.f));
         }
-        const uint32_t buf = stage + (uint32_t)(qq & 1) * kStageBuf;
-        if (storer) bulk_wait_read1();                    // stores of quarter k-2 have read `buf`
+        const uint32_t buf = stage + (uint32_t)qs * kStageBuf;
+        if (++qs == NSTG) qs = 0;
+        if (storer) bulk_wait_read<NSTG - 1>();           // stores of quarter k-NSTG have read `buf`
         hd::named_bar(1, kEpiWarps * 32);
 #pragma unroll
         for (int x = 0; x < 16; x += 4)
