@@ -82,8 +82,10 @@ typedef struct {
 #define TBS_HIST_FORCE_PASSES 0x200u  /* SDH: bucket-range passes with one smem copy (tests)   */
 /* SDH / 2PCF: fused multi-GPU combine (the paper's multi-GPU future work,
  * L1254-1256). Instead of writing hist / count, the call accumulates its (row-range) partial in
- * a local device buffer and, as its last kernel, adds that partial with system-scope atomics
- * into EACH of args->out_peers[0 .. n_out_peers) — uint64 [out_peer_words] device buffers,
+ * a local device buffer and adds that partial with system-scope atomics into EACH of
+ * args->out_peers[0 .. n_out_peers) — inside the pair kernel itself (its last CTA to finish,
+ * for single-launch output stages: smem-copy SDH, 2PCF) or, after multi-launch stages (bucket
+ * passes, global partials, the small fused path), in one extra kernel — uint64 [out_peer_words] device buffers,
  * out_peer_words = nb (SDH) or 1 (2PCF): the local rank's own and the other ranks' mapped over
  * NVLink by CUDA IPC (tbs_peer_open; peers need native atomics, tbs_peer_atomics_ok). That is
  * out_peer_words x n_out_peers remote adds per rank. Nothing is zeroed: the caller zeroes

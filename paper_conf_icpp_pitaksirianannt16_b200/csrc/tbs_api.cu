@@ -173,7 +173,7 @@ int D_of(const tbs_args* a) { return a->dim <= 3 ? 3 : 4; }
 template <class Op, int D, class C, int VSET = 0x1F>
 int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op& op, const uint32_t* bbox,
                 cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee, bool first_launch_on_scratch = true,
-                const OutSink& sink = OutSink{}) {
+                const OutSink& sink = OutSink{}, const TailPush& tail = TailPush{}) {
   // bbox may be nulled (TBS_FORCE_CLAMP); the 64-byte block always follows the SoA copy
   const uint32_t* bbox_block = reinterpret_cast<const uint32_t*>(soa + (size_t)D_of(a) * pad_rows(a->n));
   auto kern = pair_kernel<Op, D, C, VSET>;
@@ -208,7 +208,7 @@ int launch_pair(const Device& dev, const float* soa, const tbs_args* a, const Op
   static const bool trace_on = getenv("TBS_TRACE") != nullptr;  // debug: CTA residency trace to stderr
   if (trace_on) TBS_CUDA(cudaMalloc(&g.trace, (size_t)grid * 3 * 8));
   if (eb) TBS_CUDA(cudaEventRecord(eb, st));
-  kern<<<(unsigned)grid, kThreads, (size_t)smem, st>>>(soa, g, op, bbox, sink);
+  kern<<<(unsigned)grid, kThreads, (size_t)smem, st>>>(soa, g, op, bbox, sink, tail);
   TBS_CUDA(cudaGetLastError());
   g_launches.fetch_add(1);
   if (ee) TBS_CUDA(cudaEventRecord(ee, st));
@@ -377,11 +377,29 @@ OutSink local_sink(unsigned long long* buf) {
   return o;
 }
 
-// TBS_OUT_PEERS, second stage: add the local accumulator into every rank's buffer.
-int push_to_peers(const tbs_args* a, const unsigned long long* acc, int words, cudaStream_t st) {
+OutSink peer_sink(const tbs_args* a) {
   OutSink o{};
   o.n = a->n_out_peers;
   for (int w = 0; w < o.n; ++w) o.p[w] = reinterpret_cast<unsigned long long*>(a->out_peers[w]);
+  return o;
+}
+
+// TBS_OUT_PEERS in the pair kernel's tail (single-launch output stages): the last CTA pushes
+// the local accumulator `acc` (words u64) into every rank's buffer; `ticket` is a zeroed u32.
+TailPush tail_push(const tbs_args* a, const unsigned long long* acc, int words, uint32_t* ticket) {
+  TailPush t{};
+  t.peers = peer_sink(a);
+  t.acc = acc;
+  t.ticket = ticket;
+  t.words = words;
+  return t;
+}
+
+// TBS_OUT_PEERS, second stage as its own launch (multi-launch output stages: bucket-range
+// passes, global partials + reduce, the small fused path): add the local accumulator into
+// every rank's buffer.
+int push_to_peers(const tbs_args* a, const unsigned long long* acc, int words, cudaStream_t st) {
+  const OutSink o = peer_sink(a);
   push_peers<<<(words + 255) / 256, 256, 0, st>>>(acc, words, o);
   TBS_CUDA(cudaGetLastError());
   g_launches.fetch_add(1);
@@ -411,22 +429,24 @@ struct SdhPlan {
 // Lattice mode: the fast variants 4 and 0 (their own instantiation, LatFastCfg) and the
 // exact general variants 1-3 (LatCfg) are two launches; the one whose variant the bounding box does
 // not select exits at once (the work-queue counter is untouched by it).
+// (Both launches carry the fused-combine tail: only the working one takes tickets.)
 template <class Op, int D, class C, bool LAT>
 int launch_sdh(const Device& dev, const float* soa, const tbs_args* g, const Op& op, const uint32_t* bbox,
-               cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee, const OutSink& sink) {
+               cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee, const OutSink& sink, const TailPush& tail) {
   if constexpr (!LAT) {
-    return launch_pair<Op, D, C>(dev, soa, g, op, bbox, st, eb, ee, true, sink);
+    return launch_pair<Op, D, C>(dev, soa, g, op, bbox, st, eb, ee, true, sink, tail);
   } else {
-    int rc = launch_pair<Op, D, LatFastCfg, 0x11>(dev, soa, g, op, bbox, st, eb, nullptr, true, sink);
+    int rc = launch_pair<Op, D, LatFastCfg, 0x11>(dev, soa, g, op, bbox, st, eb, nullptr, true, sink, tail);
     if (rc) return rc;
-    return launch_pair<Op, D, C, 0xE>(dev, soa, g, op, bbox, st, nullptr, ee, true, sink);
+    return launch_pair<Op, D, C, 0xE>(dev, soa, g, op, bbox, st, nullptr, ee, true, sink, tail);
   }
 }
 
 template <int D, bool LAT>
 int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const uint32_t* bbox, const tbs_args* g, float w,
                  long long m, int j, int nb, const OutSink& hist, unsigned long long* part, int G, cudaStream_t st,
-                 cudaEvent_t eb, cudaEvent_t ee) {
+                 cudaEvent_t eb, cudaEvent_t ee, const TailPush& tail, bool& pushed) {
+  pushed = false;   // set when a single-launch output stage carried the fused-combine tail
   if (pl.global) {
     SdhGlobalOp<LAT> op{};
     op.nb = nb;
@@ -480,36 +500,43 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
       if constexpr (!LAT) {   // (lattice mode never takes the small-problem config)
         if (small) {
           fill(op, 32, (long long)SmallCfg::KA * SmallCfg::TP);
-          return launch_pair<SdhSmemOp<5, LAT>, D, SmallCfg>(dev, soa, g, op, bbox, st, eb, ee, true, hist);
+          pushed = tail.words > 0;
+          return launch_pair<SdhSmemOp<5, LAT>, D, SmallCfg>(dev, soa, g, op, bbox, st, eb, ee, true, hist, tail);
         }
       }
       fill(op, 32, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<5, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
+      pushed = tail.words > 0;
+      return launch_sdh<SdhSmemOp<5, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist, tail);
     }
     case 4: {
       SdhSmemOp<4, LAT> op{};
       fill(op, 16, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<4, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
+      pushed = tail.words > 0;
+      return launch_sdh<SdhSmemOp<4, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist, tail);
     }
     case 3: {
       SdhSmemOp<3, LAT> op{};
       fill(op, 8, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<3, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
+      pushed = tail.words > 0;
+      return launch_sdh<SdhSmemOp<3, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist, tail);
     }
     case 2: {
       SdhSmemOp<2, LAT> op{};
       fill(op, 4, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<2, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
+      pushed = tail.words > 0;
+      return launch_sdh<SdhSmemOp<2, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist, tail);
     }
     case 1: {
       SdhSmemOp<1, LAT> op{};
       fill(op, 2, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<1, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
+      pushed = tail.words > 0;
+      return launch_sdh<SdhSmemOp<1, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist, tail);
     }
     default: {
       SdhSmemOp<0, LAT> op{};
       fill(op, 1, (long long)C::KA * C::TP);
-      return launch_sdh<SdhSmemOp<0, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist);
+      pushed = tail.words > 0;
+      return launch_sdh<SdhSmemOp<0, LAT>, D, C, LAT>(dev, soa, g, op, bbox, st, eb, ee, hist, tail);
     }
   }
 }
@@ -618,15 +645,18 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   uint32_t* bbox = nullptr;
   rc = load_points(a, D, n_pad, &soa, pl.global ? part : h, pl.global ? zero_words : nb, st, &bbox);
   if (!rc) rc = validate_points(a, bbox, D, lattice, st);
+  // fused combine in the pair kernel's tail: ticket = the zeroed spare word 12 of the box block
+  const TailPush tail = peers && !rc ? tail_push(a, acc, nb, bbox + 12) : TailPush{};
   if (a->flags & TBS_FORCE_CLAMP) bbox = nullptr;
+  bool pushed = false;
   if (!rc) {
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
-    if (D == 3) rc = lattice ? sdh_dispatch<3, true>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee)
-                             : sdh_dispatch<3, false>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee);
-    else rc = lattice ? sdh_dispatch<4, true>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee)
-                      : sdh_dispatch<4, false>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee);
+    if (D == 3) rc = lattice ? sdh_dispatch<3, true>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee, tail, pushed)
+                             : sdh_dispatch<3, false>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee, tail, pushed);
+    else rc = lattice ? sdh_dispatch<4, true>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee, tail, pushed)
+                      : sdh_dispatch<4, false>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee, tail, pushed);
   }
-  if (!rc && peers) rc = push_to_peers(a, acc, nb, st);
+  if (!rc && peers && !pushed) rc = push_to_peers(a, acc, nb, st);
   release_soa(soa, st);
   if (part) cudaFreeAsync(part, st);
   if (acc) cudaFreeAsync(acc, st);
@@ -661,23 +691,24 @@ int pcf_impl(const tbs_args* a, float r, uint64_t* count) {
   rc = load_points(a, D, pad_rows(a->n), &soa, peers ? nullptr : c, peers ? 0 : 1, st, &bbox);
   if (!rc) rc = validate_points(a, bbox, D, false, st);
   // TBS_OUT_PEERS: the local accumulator is the zeroed spare u64 at byte 40 of the bounding-box
-  // block (words 0..2D are the box, 14-15 the work counter)
+  // block (words 0..2D are the box, 12 the fused combine's ticket, 14-15 the work counter)
   unsigned long long* acc = peers ? reinterpret_cast<unsigned long long*>(bbox + 10) : c;
   if (!rc) {
     PcfOp op{};
     op.r2 = (float)((double)r * (double)r);
     const OutSink sink = local_sink(acc);
+    // fused combine in the pair kernel's tail (ticket: the zeroed spare word 12 of the box block)
+    const TailPush tail = peers ? tail_push(a, acc, 1, bbox + 12) : TailPush{};
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
     const bool small =
         make_geom(a->n, a->row_begin, a->row_end, PcfCfg::TA, PcfCfg::TP).items < (long long)small_items_per_sm() * dev.sms;
     if (small)
-      rc = D == 3 ? launch_pair<PcfOp, 3, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink)
-                  : launch_pair<PcfOp, 4, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink);
+      rc = D == 3 ? launch_pair<PcfOp, 3, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink, tail)
+                  : launch_pair<PcfOp, 4, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink, tail);
     else
-      rc = D == 3 ? launch_pair<PcfOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink)
-                  : launch_pair<PcfOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink);
+      rc = D == 3 ? launch_pair<PcfOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink, tail)
+                  : launch_pair<PcfOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee, true, sink, tail);
   }
-  if (!rc && peers) rc = push_to_peers(a, acc, 1, st);
   release_soa(soa, st);
   return rc;
 }

@@ -227,6 +227,35 @@ struct OutSink {
   }
 };
 
+// Fused multi-GPU combine folded into the pair kernel's tail (TBS_OUT_PEERS, single-launch
+// output stages): every CTA's flush lands in the rank's local accumulator `acc` (device-scope
+// atomics); each CTA then takes a ticket, and the LAST CTA of the grid adds the `words` of
+// `acc` into every rank's buffer (`peers`, n >= 1: local or mapped from a peer GPU over
+// NVLink) with system-scope atomics — the compute and its all-reduce exchange in ONE kernel.
+// words == 0: no tail (the caller pushes with push_peers, or there are no peers).
+struct TailPush {
+  OutSink peers;
+  const unsigned long long* acc;
+  unsigned int* ticket;   // zeroed before the launch (a spare word of the bounding-box block)
+  int words;
+};
+
+__device__ __forceinline__ void push_tail(const TailPush& t) {
+  __shared__ unsigned int s_last;
+  __threadfence();        // this CTA's flush atomics are visible device-wide before its ticket
+  __syncthreads();
+  if (threadIdx.x == 0) s_last = atomicAdd(t.ticket, 1u) == gridDim.x - 1 ? 1u : 0u;
+  __syncthreads();
+  if (s_last) {
+    __threadfence();      // every other CTA's flush precedes its ticket: read acc from L2
+    for (int k = threadIdx.x; k < t.words; k += blockDim.x) {
+      const unsigned long long v = __ldcg(t.acc + k);
+      if (v) t.peers.add(k, v);
+    }
+    t.peers.fence();
+  }
+}
+
 // ------------------------------------------------------------------------------------
 // Output-stage policies. Each provides:
 //   smem_bytes()                    dynamic shared memory it needs (host and device)
@@ -754,7 +783,8 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
 template <class Op, int D, class C, int VSET = 0x1F>
 __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __restrict__ soa, Geom g, Op op,
                                                             const uint32_t* __restrict__ bbox,
-                                                            const __grid_constant__ OutSink sink) {
+                                                            const __grid_constant__ OutSink sink,
+                                                            const __grid_constant__ TailPush tail) {
   unsigned char* smem = tbs_smem;
   const long long hbytes = (op.smem_bytes() + 127) & ~127ll;
   float* bufs = reinterpret_cast<float*>(smem + hbytes);
@@ -895,6 +925,7 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
     g.trace[3 * blockIdx.x + 1] = t_start;
     g.trace[3 * blockIdx.x + 2] = t_end;
   }
+  if (tail.words > 0) push_tail(tail);   // kernel-uniform (a launch parameter)
 }
 
 // Fused multi-GPU combine, second stage (TBS_OUT_PEERS): the call's kernels accumulated this

@@ -204,6 +204,57 @@ __global__ void k_atoms_big(unsigned* out, int log2bins) {
   if (threadIdx.x == 0 && h[5] == 0xffffffffu) out[0] = h[0];
 }
 
+// Same-address degree: groups of DEG lanes share one lane-private-row word (32/DEG distinct
+// addresses per warp instruction, all in distinct banks).
+template <int DEG>
+__global__ void k_atoms_deg(unsigned* out) {
+  extern __shared__ unsigned h[];
+  const int lane = threadIdx.x & 31;
+  for (int i = threadIdx.x; i < 64 * 32; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  uint32_t a[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c)
+    a[c] = (uint32_t)__cvta_generic_to_shared(h + ((threadIdx.x * 7 + c * 13) & 63) * 32 + (lane & ~(DEG - 1)));
+  for (int i = 0; i < ITERS / 4; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(a[c]));
+  }
+  __syncthreads();
+  if (threadIdx.x == 0 && h[5] == 0xffffffffu) out[0] = h[0];
+}
+
+// ---- float -> int conversion (F2I: to confirm it must be avoided per pair) --
+__global__ void k_f2i(float* out) {
+  float x[8];
+  int acc = 0;
+#pragma unroll
+  for (int c = 0; c < 8; ++c) x[c] = 1.5f + threadIdx.x * 1e-3f + c;
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      int k;
+      asm volatile("cvt.rmi.s32.f32 %0, %1;" : "=r"(k) : "f"(x[c]));
+      acc ^= k;
+      x[c] += 0.75f;   // a new operand every iteration (FADD on the FMA pipe, beside the conversion)
+    }
+  }
+  if (acc == 12345) out[0] = (float)acc;
+}
+
+// ---- SHFL (the paper's Alg. 4 register sharing moves partners by shuffles) -------------------
+__global__ void k_shfl(float* out) {
+  float v[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) v[c] = threadIdx.x + c;
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) v[c] = __shfl_xor_sync(0xffffffffu, v[c], 1 << (c & 3));   // data stays lane-varying
+  }
+  float s = 0; for (int c = 0; c < 8; ++c) s += v[c];
+  if (s == 1.2345f) out[0] = s;
+}
+
 // ---- LDS.128 broadcast ---------------------------------------------------------
 __global__ void k_lds128(float* out) {
   __shared__ float4 s[1024];
@@ -278,6 +329,11 @@ int main() {
   atoms_big("atoms_random_16k_r1_2x256", 0, 2, 256);
   atoms_big("atoms_random_16k_r1_3x256", 0, 3, 256);
   rep("lds128_bcast_instr", (double)ITERS * thr, timeit([&] { k_lds128<<<blocks, threads>>>(dout); }));
+  rep("atoms_same_addr_deg2", at, timeit([&] { k_atoms_deg<2><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("atoms_same_addr_deg4", at, timeit([&] { k_atoms_deg<4><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("atoms_same_addr_deg8", at, timeit([&] { k_atoms_deg<8><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("f2i", it, timeit([&] { k_f2i<<<blocks, threads>>>(dout); }));
+  rep("shfl_idx_lanes", it, timeit([&] { k_shfl<<<blocks, threads>>>(dout); }));
   size_t bytes = (size_t)8 << 30; float4* big; CK(cudaMalloc(&big, bytes));
   double tw = timeit([&] { k_write<<<sms * 4, 512>>>(big, bytes / 16); });
   printf(", \"hbm_write_stcs_GBps\": %.1f", bytes / tw * 1e-9);
