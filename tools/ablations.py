@@ -41,7 +41,7 @@ n = int(os.environ.get("ABL_N", 1 << 20))
 pairs = n * (n - 1) // 2
 pu = torch.from_numpy(g.uniform(n, 2)).cuda()
 pc = torch.from_numpy(g.clustered(n, 3)).cuda()
-for nb in (16, 64, 256, 512, 768, 1024, 2048, 4096, 6144, 8192, 16384, 32768, 49152, 65536):
+for nb in (16, 64, 256, 512, 768, 1024, 2048, 4096, 6144, 8192, 16384, 32768, 49152, 65536, 98304, 131072):
     w = float(np.float32(math.sqrt(3) / nb))
     ms = timed(lambda: tbs.sdh(pu, w, nb))
     emit(ablation="nb_sweep", n=n, nb=nb, ms=ms, gpairs_s=pairs / ms / 1e6)

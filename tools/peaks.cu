@@ -204,8 +204,9 @@ __global__ void k_atoms_big(unsigned* out, int log2bins) {
   if (threadIdx.x == 0 && h[5] == 0xffffffffu) out[0] = h[0];
 }
 
-// Same-address degree: groups of DEG lanes share one lane-private-row word (32/DEG distinct
-// addresses per warp instruction, all in distinct banks).
+// Same-address degree: groups of DEG lanes share one word of a warp-uniform row (32/DEG
+// distinct addresses per warp instruction, all in distinct banks). (Bank-conflict degree DEG,
+// DEG distinct rows hit through one bank: k_atoms_bank.)
 template <int DEG>
 __global__ void k_atoms_deg(unsigned* out) {
   extern __shared__ unsigned h[];
@@ -215,7 +216,26 @@ __global__ void k_atoms_deg(unsigned* out) {
   uint32_t a[8];
 #pragma unroll
   for (int c = 0; c < 8; ++c)
-    a[c] = (uint32_t)__cvta_generic_to_shared(h + ((threadIdx.x * 7 + c * 13) & 63) * 32 + (lane & ~(DEG - 1)));
+    a[c] = (uint32_t)__cvta_generic_to_shared(h + (((threadIdx.x >> 5) * 7 + c * 13) & 63) * 32 + (lane & ~(DEG - 1)));
+  for (int i = 0; i < ITERS / 4; ++i) {
+#pragma unroll
+    for (int c = 0; c < 8; ++c) asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(a[c]));
+  }
+  __syncthreads();
+  if (threadIdx.x == 0 && h[5] == 0xffffffffu) out[0] = h[0];
+}
+
+template <int DEG>
+__global__ void k_atoms_bank(unsigned* out) {
+  extern __shared__ unsigned h[];
+  const int lane = threadIdx.x & 31;
+  for (int i = threadIdx.x; i < 64 * 32; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  uint32_t a[8];
+#pragma unroll
+  for (int c = 0; c < 8; ++c)   // lanes of a group: the same bank (column), different rows
+    a[c] = (uint32_t)__cvta_generic_to_shared(h + (((threadIdx.x >> 5) * 7 + c * 13 + (lane & (DEG - 1))) & 63) * 32 +
+                                              (lane & ~(DEG - 1)));
   for (int i = 0; i < ITERS / 4; ++i) {
 #pragma unroll
     for (int c = 0; c < 8; ++c) asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(a[c]));
@@ -332,6 +352,10 @@ int main() {
   rep("atoms_same_addr_deg2", at, timeit([&] { k_atoms_deg<2><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
   rep("atoms_same_addr_deg4", at, timeit([&] { k_atoms_deg<4><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
   rep("atoms_same_addr_deg8", at, timeit([&] { k_atoms_deg<8><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("atoms_same_addr_deg16", at, timeit([&] { k_atoms_deg<16><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("atoms_bank_conflict_deg2", at, timeit([&] { k_atoms_bank<2><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("atoms_bank_conflict_deg4", at, timeit([&] { k_atoms_bank<4><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
+  rep("atoms_bank_conflict_deg8", at, timeit([&] { k_atoms_bank<8><<<blocks, threads, 64 * 32 * 4>>>((unsigned*)dout); }));
   rep("f2i", it, timeit([&] { k_f2i<<<blocks, threads>>>(dout); }));
   rep("shfl_idx_lanes", it, timeit([&] { k_shfl<<<blocks, threads>>>(dout); }));
   size_t bytes = (size_t)8 << 30; float4* big; CK(cudaMalloc(&big, bytes));
