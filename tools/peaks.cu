@@ -342,6 +342,27 @@ int main() {
     if (log2r == 1) rep(name, ops, timeit([&] { k_atoms_big<1><<<sms * cta_per_sm, thr_per_cta, sm_b>>>((unsigned*)dout, 14); }));
     else rep(name, ops, timeit([&] { k_atoms_big<0><<<sms * cta_per_sm, thr_per_cta, sm_b>>>((unsigned*)dout, 14); }));
   };
+  // windows of fewer bins with more replicas (what a spatially sorted tile pair would allow)
+  auto atoms_win = [&](const char* name, int log2bins, int log2r, int cta_per_sm, int thr_per_cta) {
+    const double ops = (double)(ITERS / 4) * 8 * sms * cta_per_sm * thr_per_cta;
+    const size_t sm_b = ((size_t)4 << log2bins) << log2r;
+    auto go = [&](auto kern) {
+      CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_b));
+      rep(name, ops, timeit([&] { kern<<<sms * cta_per_sm, thr_per_cta, sm_b>>>((unsigned*)dout, log2bins); }));
+      return 0;
+    };
+    if (log2r == 2) go(k_atoms_big<2>);
+    if (log2r == 3) go(k_atoms_big<3>);
+    if (log2r == 4) go(k_atoms_big<4>);
+    if (log2r == 5) go(k_atoms_big<5>);
+  };
+  atoms_win("atoms_random_8k_r4_1x256", 13, 2, 1, 256);
+  atoms_win("atoms_random_4k_r8_1x256", 12, 3, 1, 256);
+  atoms_win("atoms_random_4k_r8_1x512", 12, 3, 1, 512);
+  atoms_win("atoms_random_2k_r16_1x256", 11, 4, 1, 256);
+  atoms_win("atoms_random_2k_r16_1x512", 11, 4, 1, 512);
+  atoms_win("atoms_random_1k_r32_1x512", 10, 5, 1, 512);
+  atoms_win("atoms_random_1k_r32_2x256", 10, 5, 2, 256);
   atoms_big("atoms_random_16k_r2_1x256", 1, 1, 256);
   atoms_big("atoms_random_16k_r2_1x512", 1, 1, 512);
   atoms_big("atoms_random_16k_r2_1x1024", 1, 1, 1024);
