@@ -93,7 +93,13 @@ using LatFastCfg = Cfg<TBS_LATF_CFG>;
 #ifndef TBS_SMALL_TP
 #define TBS_SMALL_TP 128
 #endif
-using SmallCfg = Cfg<2, TBS_SMALL_TP, 4>;
+#ifndef TBS_SMALL_KA
+#define TBS_SMALL_KA 2
+#endif
+#ifndef TBS_SMALL_MINB
+#define TBS_SMALL_MINB 4
+#endif
+using SmallCfg = Cfg<TBS_SMALL_KA, TBS_SMALL_TP, TBS_SMALL_MINB>;
 // Use the small-problem config when the main config yields fewer than this many items per SM.
 int small_items_per_sm() {
   static const int v = [] { const char* e = getenv("TBS_SMALL_ITEMS"); return e ? atoi(e) : 16; }();
