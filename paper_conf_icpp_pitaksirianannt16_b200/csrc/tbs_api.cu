@@ -335,7 +335,7 @@ int load_points(const tbs_args* a, int D, int n_pad, float** soa, unsigned long 
   } else {
     TBS_CUDA(cudaMemsetAsync(*bbox, 0, 64, st));
     const int threads = 256;
-    long long blocks = std::min<long long>((n_pad + threads - 1) / threads, 148ll * 16);
+    long long blocks = std::min<long long>((n_pad + threads - 1) / threads, 148ll * 8);
     blocks = std::max<long long>(blocks, 1);
     soa_loader<<<(unsigned)blocks, threads, 0, st>>>(a->points, (int)a->n, a->dim, n_pad, D, pad, *soa, zero,
                                                      zero_words, *bbox);

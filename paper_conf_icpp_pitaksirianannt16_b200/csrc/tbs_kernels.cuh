@@ -119,6 +119,11 @@ __global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_
   }
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < zero_words; i += stride) zero[i] = 0ull;
   if (bbox) {
+    // warp shuffles, then the CTA's warps in shared memory, then ONE atomic per box word per
+    // CTA (per-warp global atomics on the same 2D+1 words serialised in L2: ~0.1 ms at 1M)
+    __shared__ uint32_t sb[9];
+    if (threadIdx.x < 9) sb[threadIdx.x] = 0u;
+    __syncthreads();
     for (int c = 0; c < D; ++c) {
       uint32_t a = lo[c], b = hi[c];
 #pragma unroll
@@ -127,13 +132,19 @@ __global__ void soa_loader(const float* __restrict__ pts, int n, int dim, int n_
         b = max(b, __shfl_xor_sync(0xffffffffu, b, off));
       }
       if ((threadIdx.x & 31) == 0) {
-        if (a) atomicMax(bbox + c, a);
-        if (b) atomicMax(bbox + D + c, b);
+        if (a) atomicMax(sb + c, a);
+        if (b) atomicMax(sb + D + c, b);
       }
     }
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) bad |= __shfl_xor_sync(0xffffffffu, bad, off);
-    if ((threadIdx.x & 31) == 0 && bad) atomicOr(bbox + 2 * D, bad);
+    if ((threadIdx.x & 31) == 0 && bad) atomicOr(sb + 2 * D, bad);
+    __syncthreads();
+    if (threadIdx.x < 2 * D) {
+      if (sb[threadIdx.x]) atomicMax(bbox + threadIdx.x, sb[threadIdx.x]);
+    } else if (threadIdx.x == 2 * D && sb[2 * D]) {
+      atomicOr(bbox + 2 * D, sb[2 * D]);
+    }
   }
 }
 
