@@ -31,6 +31,10 @@ namespace tbs {
 constexpr int kThreads = 256;              // 8 warps per CTA
 constexpr int kPUnroll = TBS_PUNROLL;
 constexpr unsigned kSwSqrtMask = TBS_SW_SQRT;
+#ifndef TBS_MQ_ORDER
+#define TBS_MQ_ORDER 0                     // A/B only: 1 = anchor-major slots for every Op; 2, 3 = two-phase groups
+#endif
+constexpr int kMqOrder = TBS_MQ_ORDER;
 #ifndef TBS_PARTNER_PATH
 #define TBS_PARTNER_PATH 0                 // Fig. 9 ablation (A/B builds only): how partners reach the
 #endif                                     // threads, see run_chunk
@@ -425,6 +429,9 @@ struct SdhSmemOp {
 
   // Float mode, unmasked pairs, square roots on the FMA pipe (the TBS_SW_SQRT slots).
   static constexpr bool kSwCapable = !LATTICE && !RANGED;
+  // slot order of a partner group (run_chunk): anchor-major measured +1.0 % for float SDH at
+  // 1M, but -7.4 % for the lattice variants at 4M (profiles/r02_slot_order_ab.txt)
+  static constexpr bool kAnchorMajor = !LATTICE;
   template <int V>
   __device__ __forceinline__ void pair2_sw(float2 s) {
     uint32_t ad0, ad1;
@@ -565,6 +572,7 @@ struct SdhGlobalOp {
   const OutSink* out;        // unused (the reduce kernel writes the sink)
 
   static constexpr bool kSwCapable = false;
+  static constexpr bool kAnchorMajor = false;   // slot order (run_chunk; r02 A/B)
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) { mine = part + (size_t)(blockIdx.x % G) * nb; }
   __device__ __forceinline__ float2 bias() const { return make_float2(0.f, 0.f); }
@@ -610,6 +618,7 @@ struct PcfOp {
   uint32_t c;                // per-item counter (<= KA * TP)
   unsigned long long total;  // per-thread running total
   static constexpr bool kSwCapable = false;
+  static constexpr bool kAnchorMajor = false;   // slot order (run_chunk; r02 A/B)
 
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) { c = 0u; total = 0ull; }
@@ -659,6 +668,7 @@ struct KdeOp {
   float tot, comp;          // Kahan running sum
   const OutSink* out;       // unused
   static constexpr bool kSwCapable = false;
+  static constexpr bool kAnchorMajor = true;   // slot order (run_chunk; r02 A/B)
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) {
     part = make_float2(0.f, 0.f);
@@ -762,12 +772,43 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
 #pragma unroll
         for (int q = 0; q < 4; ++q) c4[c][q] = __shfl_sync(0xffffffffu, sh[c], (p & 31) + q);
     }
+    if constexpr (kMqOrder >= 2 && !(Op::kSwCapable && kSwSqrtMask != 0u)) {
+      // A/B: two phases over PH slots (anchor-major): all squared distances, then all outputs
+      constexpr int NS = 4 * (C::KA / 2), PH = kMqOrder == 2 ? NS : 4;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
+      for (int base = 0; base < NS; base += PH) {
+        float2 sv[PH];
+#pragma unroll
+        for (int j = 0; j < PH; ++j) {
+          const int q = (base + j) % 4, m = (base + j) / 4;
+          float2 d = __fadd2_rn(na[0][m], make_float2(c4[0][q], c4[0][q]));
+          sv[j] = __ffma2_rn(d, d, op.bias());
+#pragma unroll
+          for (int c = 1; c < D; ++c) {
+            d = __fadd2_rn(na[c][m], make_float2(c4[c][q], c4[c][q]));
+            sv[j] = __ffma2_rn(d, d, sv[j]);
+          }
+        }
+#pragma unroll
+        for (int j = 0; j < PH; ++j) {
+          const int q = (base + j) % 4, m = (base + j) / 4;
+          const int pv = MASKED ? ((p0 + p + q < n) ? p0 + p + q : -1) : 0;
+          op.template pair2<MASKED, V>(sv[j], pv, MASKED ? aidx[2 * m] : 0, MASKED ? aidx[2 * m + 1] : 0);
+        }
+      }
+      op.after_group();
+      continue;
+    }
+#pragma unroll
+    for (int qm = 0; qm < 4 * (C::KA / 2); ++qm) {
+      // partner q, anchor pair m: partner-major or anchor-major — the order ptxas schedules the
+      // 4 x KA/2 independent chains in (per Op, measured; TBS_MQ_ORDER=1 forces anchor-major)
+      constexpr bool am = Op::kAnchorMajor || kMqOrder == 1;
+      const int q = am ? qm % 4 : qm / (C::KA / 2);
+      const int m = am ? qm / 4 : qm % (C::KA / 2);
       int pv = 0;
       if (MASKED) pv = (p0 + p + q < n) ? p0 + p + q : -1;
-#pragma unroll
-      for (int m = 0; m < C::KA / 2; ++m) {
+      {
         float2 d = __fadd2_rn(na[0][m], make_float2(c4[0][q], c4[0][q]));
         float2 s = __ffma2_rn(d, d, op.bias());
 #pragma unroll
