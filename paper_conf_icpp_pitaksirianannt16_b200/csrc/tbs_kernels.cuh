@@ -804,8 +804,18 @@ __device__ __forceinline__ void run_chunk(Op& op, const float* __restrict__ B, c
       // partner q, anchor pair m: partner-major or anchor-major — the order ptxas schedules the
       // 4 x KA/2 independent chains in (per Op, measured; TBS_MQ_ORDER=1 forces anchor-major)
       constexpr bool am = Op::kAnchorMajor || kMqOrder == 1;
-      const int q = am ? qm % 4 : qm / (C::KA / 2);
-      const int m = am ? qm / 4 : qm % (C::KA / 2);
+      constexpr int M = C::KA / 2;
+      int q = am ? qm % 4 : qm / M;
+      int m = am ? qm / 4 : qm % M;
+      if constexpr (kMqOrder == 4 && M % 2 == 0) {   // A/B: 2 x 2 blocks (anchor pairs x partners)
+        const int blk = qm / 4, in = qm % 4;
+        m = (blk / 2) * 2 + in / 2;
+        q = (blk % 2) * 2 + in % 2;
+      }
+      if constexpr (kMqOrder == 5) {                  // A/B: diagonal
+        m = qm % M;
+        q = (qm / M + qm % M) % 4;
+      }
       int pv = 0;
       if (MASKED) pv = (p0 + p + q < n) ? p0 + p + q : -1;
       {
