@@ -80,12 +80,6 @@ typedef struct {
 #define TBS_HIST_FORCE_GLOBAL 0x40u   /* SDH: partially privatised global u64 copies       */
 #define TBS_FORCE_CLAMP 0x100u        /* SDH: never elide the nb-1 clamp (ablation/tests)   */
 #define TBS_HIST_FORCE_PASSES 0x200u  /* SDH: bucket-range passes with one smem copy (tests)   */
-/* SDH, float mode, full row range, n >= 2: the windowed stage (points ordered in space, each
- * work item counted in a window of buckets with more replicas; large nb) even where the
- * automatic choice would not take it (tests, A/B). Ignored where it does not apply. */
-#define TBS_HIST_FORCE_WINDOW 0x1000u
-/* SDH: never the windowed stage. */
-#define TBS_HIST_NO_WINDOW 0x2000u
 /* SDH / 2PCF: fused multi-GPU combine (the paper's multi-GPU future work,
  * L1254-1256). Instead of writing hist / count, the call accumulates its (row-range) partial in
  * a local device buffer and adds that partial with system-scope atomics into EACH of

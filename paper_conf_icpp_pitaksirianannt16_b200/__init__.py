@@ -36,12 +36,10 @@ TBS_FORCE_CLAMP = 0x100
 TBS_HIST_FORCE_PASSES = 0x200
 TBS_OUT_PEERS = 0x400
 TBS_VALIDATE = 0x800
-TBS_HIST_FORCE_WINDOW = 0x1000
-TBS_HIST_NO_WINDOW = 0x2000
 TBS_MAX_PEERS = 16
 KERNELS = {"gaussian": 0, "dist2": 1, "dist": 2}
 HIST_MODES = {None: 0, "lane": TBS_HIST_FORCE_LANE, "cta": TBS_HIST_FORCE_CTA, "global": TBS_HIST_FORCE_GLOBAL,
-              "passes": TBS_HIST_FORCE_PASSES, "window": TBS_HIST_FORCE_WINDOW, "nowindow": TBS_HIST_NO_WINDOW}
+              "passes": TBS_HIST_FORCE_PASSES}
 
 # Symbols declared in include/tbs.h (checked by tests/test_abi.py).
 EXPORTS = ("tbs_sdh", "tbs_pcf", "tbs_pairmatrix", "tbs_sdh_ex", "tbs_pcf_ex", "tbs_pairmatrix_ex",

@@ -22,7 +22,6 @@
 #include "tbs_hd2.cuh"
 #include "tbs_knn.cuh"
 #include "tbs_rdf.cuh"
-#include "tbs_win.cuh"
 
 using namespace tbs;
 static_assert(kMaxPeers == TBS_MAX_PEERS, "peer sink size");
@@ -101,20 +100,6 @@ using LatFastCfg = Cfg<TBS_LATF_CFG>;
 #define TBS_SMALL_MINB 4
 #endif
 using SmallCfg = Cfg<TBS_SMALL_KA, TBS_SMALL_TP, TBS_SMALL_MINB>;
-// Windowed large-nb SDH (tbs_win.cuh): replicas per window bucket, anchors per thread, chunk.
-#ifndef TBS_WIN_LOG2R
-#define TBS_WIN_LOG2R 4
-#endif
-#ifndef TBS_WIN_KA
-#define TBS_WIN_KA 4
-#endif
-#ifndef TBS_WIN_TP
-#define TBS_WIN_TP 512
-#endif
-#ifndef TBS_WIN_MINB
-#define TBS_WIN_MINB 1
-#endif
-using WinCfg = Cfg<TBS_WIN_KA, TBS_WIN_TP, TBS_WIN_MINB>;
 // Use the small-problem config when the main config yields fewer than this many items per SM.
 int small_items_per_sm() {
   static const int v = [] { const char* e = getenv("TBS_SMALL_ITEMS"); return e ? atoi(e) : 16; }();
@@ -562,62 +547,6 @@ int sdh_dispatch(const Device& dev, const SdhPlan& pl, const float* soa, const u
   }
 }
 
-// Windowed stage (full-range float SDH with large nb): order the points in space (counting sort
-// by Morton cell over the loader's box), box every TP-point chunk, then one pair-kernel launch
-// whose items count into a per-item window of buckets with 2^TBS_WIN_LOG2R replicas.
-int sdh_windowed(const Device& dev, const tbs_args* a, const float* soa, const uint32_t* bbox, float w, int nb,
-                 const OutSink& sink, const TailPush& tail, cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee) {
-  using C = WinCfg;
-  const int n = (int)a->n, n_pad = pad_rows(a->n);
-  int g = 1;   // grid 2^g per dimension, ~32 points per cell on average, at most 2^18 cells
-  while (g < 6 && (8ll << (3 * (g + 1))) * 4 <= (long long)n) ++g;
-  const int ncells = 1 << (3 * g);
-  const int nchunks = (n + C::TP - 1) / C::TP + C::RATIO;   // + anchor-tile chunks past n
-  const size_t soa_bytes = (size_t)3 * n_pad * 4;
-  unsigned char* scratch = nullptr;
-  const size_t bytes = soa_bytes + 64 + (size_t)n * 4 + (size_t)ncells * 4 + (size_t)nchunks * 24;
-  TBS_CUDA(cudaMallocAsync((void**)&scratch, bytes, st));
-  float* soa2 = reinterpret_cast<float*>(scratch);
-  uint32_t* cell = reinterpret_cast<uint32_t*>(scratch + soa_bytes + 64);
-  uint32_t* count = cell + n;
-  float* boxes = reinterpret_cast<float*>(count + ncells);
-  int rc = TBS_OK;
-  // pads (i >= n) stay 0 like the loader's; the 64-byte block after the copy holds the work counter
-  TBS_CUDA(cudaMemsetAsync(soa2, 0, soa_bytes + 64, st));
-  TBS_CUDA(cudaMemsetAsync(count, 0, (size_t)ncells * 4, st));
-  const int blocks = std::min((n + 255) / 256, dev.sms * 8);
-  win::cell_count<<<blocks, 256, 0, st>>>(soa, n, n_pad, bbox, g, cell, count);
-  win::scan_exclusive<<<1, 1024, 0, st>>>(count, ncells);
-  win::scatter_cells<<<blocks, 256, 0, st>>>(soa, n, n_pad, cell, count, soa2);
-  win::chunk_boxes<<<nchunks, 256, 0, st>>>(soa2, n, n_pad, C::TP, boxes);
-  if (cudaGetLastError() != cudaSuccess) rc = fail(TBS_ECUDA, "windowed SDH: ordering kernels failed to launch");
-  g_launches.fetch_add(4);
-  if (!rc) {
-    SdhSmemOp<TBS_WIN_LOG2R, false, true, true> op{};
-    constexpr int Rw = 1 << TBS_WIN_LOG2R;
-    // per CTA: the SM's 228 KB shared by MINB CTAs (1 KB reserved each), minus the partner
-    // double buffer and 2 KB for the kernel's static shared memory (item slots, tail ticket)
-    const long long per_cta = std::min<long long>(dev.smem_optin, 233472 / C::MINB - 1024);
-    const long long budget = per_cta - 2ll * 3 * C::TP * 4 - 2048;
-    op.nb = nb;
-    op.rows = (int)std::min<long long>(budget / (Rw * 4) - 1, (long long)nb + kGuard);
-    op.inv_w = (float)(1.0 / (double)w);
-    op.boxes = boxes;
-    op.flush_every = 0x7fffffff;
-    op.ymax = 0.f;
-    rc = launch_pair<decltype(op), 3, C, 0x1>(dev, soa2, a, op, bbox, st, eb, ee, true, sink, tail);
-  }
-  cudaFreeAsync(scratch, st);
-  return rc;
-}
-
-constexpr bool kWinDefault = false;   // (set after the A/B: profiles/r02_win_ab.txt)
-// TBS_WIN: -1 (unset) = the windowed stage when it applies, 0 = never, 1 = whenever possible
-int win_mode() {
-  static const int v = [] { const char* e = getenv("TBS_WIN"); return e ? atoi(e) : -1; }();
-  return v;
-}
-
 int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   int rc = validate_common(a, nb);
   if (rc) return rc;
@@ -726,18 +655,7 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   const TailPush tail = peers && !rc ? tail_push(a, acc, nb, bbox + 12) : TailPush{};
   if (a->flags & TBS_FORCE_CLAMP) bbox = nullptr;
   bool pushed = false;
-  // windowed stage: full-range float SDH whose plan is <= 2 smem copies or bucket passes
-  const uint32_t forced = TBS_HIST_FORCE_LANE | TBS_HIST_FORCE_CTA | TBS_HIST_FORCE_PASSES | TBS_HIST_FORCE_GLOBAL | TBS_FORCE_CLAMP;
-  const bool win_req = (a->flags & TBS_HIST_FORCE_WINDOW) || win_mode() == 1 ||
-                       (kWinDefault && win_mode() != 0 && !(a->flags & TBS_HIST_NO_WINDOW) && !(a->flags & forced) &&
-                        a->n >= 65536 && !pl.global && pl.log2r <= 1);
-  const bool win = win_req && !rc && !lattice && D == 3 && a->row_begin == 0 && a->row_end == a->n &&
-                   !(a->flags & TBS_FORCE_CLAMP) && !(a->flags & TBS_HIST_NO_WINDOW);
-  if (win) {
-    cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
-    rc = sdh_windowed(dev, a, soa, bbox, w, nb, sink, tail, st, eb, ee);
-    pushed = tail.words > 0;
-  } else if (!rc) {
+  if (!rc) {
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
     if (D == 3) rc = lattice ? sdh_dispatch<3, true>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee, tail, pushed)
                              : sdh_dispatch<3, false>(dev, pl, soa, bbox, a, w, m, j, nb, sink, part, G, st, eb, ee, tail, pushed);

@@ -300,18 +300,10 @@ extern __shared__ __align__(128) unsigned char tbs_smem[];  // dynamic smem; his
 // RANGED: bucket-range pass for nb beyond one shared-memory copy: only buckets
 // [klo, klo + rows) are counted in this launch (one predicated ATOMS); the host runs
 // ceil(nb / rows) passes over the triangle instead of falling back to global atomics.
-// WIN (with RANGED): the windowed stage (tbs_win.cuh) — buckets [klo, klo + rows) of the current
-// work item, klo set per item (segment) from the boxes of its anchor tile and partner chunk; code
-// variant 0 = the item's whole interval fits the window (no range check, no clamp: buckets >= nb
-// fold into nb - 1 at the flush), 1 = one of several segments (range check, out-of-window pairs
-// to the trash row).
-template <int LOG2R, bool LATTICE, bool RANGED = false, bool WIN = false>
+template <int LOG2R, bool LATTICE, bool RANGED = false>
 struct SdhSmemOp {
   static constexpr int R = 1 << LOG2R;
-  static constexpr bool kWin = WIN;
-  int klo = 0;        // first bucket of this pass (RANGED) / window segment (WIN)
-  const float* boxes = nullptr;   // WIN: [chunks][lo3 hi3] of the ordered SoA (TP-point chunks)
-  int used = 0;                   // WIN: rows of the current segment that can be non-zero
+  int klo = 0;        // first bucket of this pass (RANGED)
   int nb;             // buckets
   int rows;           // rows allocated (nb, + kGuard in float mode)
   float inv_w;        // fp32(1 / w)                       (float mode)
@@ -343,7 +335,6 @@ struct SdhSmemOp {
   static constexpr int kVariants = LATTICE ? 5 : 2;
   float mj;           // lattice: m * 2^-j (exact)
   __device__ __forceinline__ int variant(const uint32_t* bbox, int D) const {
-    if (WIN) return 0;   // (per-item variants, chosen in the item loop)
     const float dmax = bbox_diameter(bbox, D);
     if (LATTICE) {
       const double smax = (double)dmax * (double)dmax;             // >= every s (integer data)
@@ -417,7 +408,7 @@ struct SdhSmemOp {
   __device__ __forceinline__ void float_addr2(float2 q, uint32_t& ad0, uint32_t& ad1, bool& in0, bool& in1) const {
     const float c = LATTICE ? scale_b : inv_w;
     float2 y = __ffma2_rd(q, make_float2(c, c), make_float2(kMagicF, kMagicF));
-    if (!LATTICE && V == 1 && !WIN) {
+    if (!LATTICE && V == 1) {
       y.x = fminf(y.x, ymax);
       y.y = fminf(y.y, ymax);
     }
@@ -430,7 +421,7 @@ struct SdhSmemOp {
     const uint32_t ub = smem_addr(tbs_smem) - ((kMagic + (RANGED ? (uint32_t)klo : 0u)) << S);
     ad0 = __funnelshift_l(lo, __float_as_uint(y.x), S) + ub;
     ad1 = __funnelshift_l(lo, __float_as_uint(y.y), S) + ub;
-    if (RANGED && !(WIN && V == 0)) {
+    if (RANGED) {
       in0 = __float_as_uint(y.x) - (kMagic + (uint32_t)klo) < (uint32_t)rows;
       in1 = __float_as_uint(y.y) - (kMagic + (uint32_t)klo) < (uint32_t)rows;
     }
@@ -494,7 +485,7 @@ struct SdhSmemOp {
       ad0 = (k0 << (LOG2R + 2)) + lb;
       ad1 = (k1 << (LOG2R + 2)) + lb;
     }
-    if ((RANGED && !(WIN && V == 0)) || MASKED) {
+    if (RANGED || MASKED) {
       // Masked pairs (i >= j, pad partners: their distance can leave the histogram) and
       // out-of-pass buckets increment the lane's word of the trash row `rows` instead: no
       // branch (a predicated ATOMS becomes BSSY/BRA/BSYNC), the same ATOMS.POPC.INC, and the
@@ -521,8 +512,7 @@ struct SdhSmemOp {
     uint32_t* h = reinterpret_cast<uint32_t*>(smem);
     const int t = threadIdx.x & 31;
     const int rot = t >> (5 - LOG2R);
-    const int lim = WIN ? used : rows;
-    for (int k = threadIdx.x; k < lim; k += kThreads) {
+    for (int k = threadIdx.x; k < rows; k += kThreads) {
       unsigned long long v = 0;
 #pragma unroll 8
       for (int j = 0; j < R; ++j) {
@@ -536,45 +526,6 @@ struct SdhSmemOp {
       }
     }
   }
-  // WIN: the bucket interval [kmin, kmax] of every pair of anchor tile I (chunks I*ratio ..
-  // +ratio-1) x partner chunk J from their boxes, in fp32 with directed rounding and a margin
-  // (2^-16 relative + 2 buckets) far above the pair kernel's own rounding (~4e-7): the kernel's
-  // bucket of any pair of the item lies inside. Non-finite boxes give [0, nb + kGuard).
-  __device__ void window(int I, int J, int ratio, int& kmin, int& kmax) const {
-    float alo[3], ahi[3];
-#pragma unroll
-    for (int c = 0; c < 3; ++c) {
-      alo[c] = __int_as_float(0x7f800000);
-      ahi[c] = -__int_as_float(0x7f800000);
-    }
-    for (int r = 0; r < ratio; ++r) {
-      const float* b = boxes + (long long)(I * ratio + r) * 6;
-#pragma unroll
-      for (int c = 0; c < 3; ++c) {
-        alo[c] = fminf(alo[c], b[c]);
-        ahi[c] = fmaxf(ahi[c], b[3 + c]);
-      }
-    }
-    const float* bj = boxes + (long long)J * 6;
-    float lo2 = 0.f, hi2 = 0.f;
-#pragma unroll
-    for (int c = 0; c < 3; ++c) {
-      const float gap = fmaxf(0.f, fmaxf(__fsub_rd(alo[c], bj[3 + c]), __fsub_rd(bj[c], ahi[c])));
-      const float span = fmaxf(__fsub_ru(bj[3 + c], alo[c]), __fsub_ru(ahi[c], bj[c]));
-      lo2 = __fmaf_rd(gap, gap, lo2);
-      hi2 = __fmaf_ru(span, span, hi2);
-    }
-    const float kl = __fmul_rd(__fmul_rd(__fsqrt_rd(lo2), inv_w), 1.f - 1.f / 65536.f);
-    const float kh = __fmul_ru(__fmul_ru(__fsqrt_ru(hi2), inv_w), 1.f + 1.f / 65536.f);
-    if (!(kl >= 0.f) || !(kh < 1.0e9f)) {
-      kmin = 0;
-      kmax = nb + kGuard - 1;
-      return;
-    }
-    kmin = max(0, (int)kl - 2);
-    kmax = (int)kh + 2;
-  }
-
   // Mid-kernel overflow flush: segmented shuffle-sum of each bin's R replicas (warp-uniform
   // loop, so the item loop around it keeps its uniform registers).
   __device__ void flush_in_loop(unsigned char* smem) {
@@ -621,7 +572,6 @@ struct SdhGlobalOp {
   const OutSink* out;        // unused (the reduce kernel writes the sink)
 
   static constexpr bool kSwCapable = false;
-  static constexpr bool kWin = false;
   static constexpr bool kAnchorMajor = false;   // slot order (run_chunk; r02 A/B)
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) { mine = part + (size_t)(blockIdx.x % G) * nb; }
@@ -668,7 +618,6 @@ struct PcfOp {
   uint32_t c;                // per-item counter (<= KA * TP)
   unsigned long long total;  // per-thread running total
   static constexpr bool kSwCapable = false;
-  static constexpr bool kWin = false;
   static constexpr bool kAnchorMajor = false;   // slot order (run_chunk; r02 A/B)
 
   __host__ __device__ long long smem_bytes() const { return 0; }
@@ -719,7 +668,6 @@ struct KdeOp {
   float tot, comp;          // Kahan running sum
   const OutSink* out;       // unused
   static constexpr bool kSwCapable = false;
-  static constexpr bool kWin = false;
   static constexpr bool kAnchorMajor = true;   // slot order (run_chunk; r02 A/B)
   __host__ __device__ long long smem_bytes() const { return 0; }
   __device__ __forceinline__ void init(unsigned char*) {
@@ -928,15 +876,6 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
   // publishes it through a parity-double-buffered shared slot.
   __shared__ long long s_it[2];
   __shared__ int s_I[2], s_J[2];
-  __shared__ int s_kmin[2], s_kmax[2];   // WIN: the item's bucket interval
-  auto publish_window = [&](int I_, int J_, int slot) {
-    if constexpr (Op::kWin) {
-      int a, b;
-      op.window(I_, J_, C::RATIO, a, b);
-      s_kmin[slot] = a;
-      s_kmax[slot] = b;
-    }
-  };
   long long it, chunk_end = 0;
   int I = 0, J = 0;
   // g.chunk == 0: one item per CTA (grid == items, small problems): item = blockIdx.x, no queue
@@ -946,7 +885,6 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
       chunk_end = g.chunk > 0 ? min(it + g.chunk, g.items) : it + 1;
       item_to_tile(g, it, I, J);
       if (kPartnerPath == 0) issue_chunk<D, C::TP>(soa, g, J, bufs, bar0);
-      publish_window(I, J, 0);
     }
     s_it[0] = it; s_I[0] = I; s_J[0] = J;
   }
@@ -972,7 +910,6 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
           }
         }
         if (kPartnerPath == 0 && nit < g.items) issue_chunk<D, C::TP>(soa, g, nJ, bufs + (s ^ 1) * D * C::TP, s ? bar0 : bar1);
-        if (nit < g.items) publish_window(nI, nJ, s ^ 1);
         s_it[s ^ 1] = nit; s_I[s ^ 1] = nI; s_J[s ^ 1] = nJ;
       }
       if (I != curI) {
@@ -996,26 +933,6 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel(const float* __
       const int cnt = min(C::TP, g.n - p0);
       const bool fast =
           (I * C::TA >= g.rb) && ((I + 1) * C::TA <= g.re) && (p0 >= (I + 1) * C::TA) && (cnt == C::TP);
-      if constexpr (Op::kWin) {
-        // windowed stage: the item's bucket interval in window segments, each flushed
-        const int kmin = s_kmin[s], kmax = s_kmax[s];
-        const int nseg = (kmax - kmin) / op.rows + 1;
-        for (int sg = 0; sg < nseg; ++sg) {
-          op.klo = kmin + sg * op.rows;
-          op.used = min(op.rows, kmax - op.klo + 1);   // rows past the item's last bucket stay zero
-          if (nseg == 1) {
-            if (fast) run_chunk<Op, D, C, false, 0>(op, B, na, g, I, p0, cnt);
-            else run_chunk<Op, D, C, true, 0>(op, B, na, g, I, p0, cnt);
-          } else {
-            if (fast) run_chunk<Op, D, C, false, 1>(op, B, na, g, I, p0, cnt);
-            else run_chunk<Op, D, C, true, 1>(op, B, na, g, I, p0, cnt);
-          }
-          __syncthreads();
-          op.flush(smem);
-          __syncthreads();
-        }
-        goto item_done;
-      }
       if constexpr (Op::kVariants > 4 && (VSET & 16)) {
         if (variant == 4) {
           if (fast) run_chunk<Op, D, C, false, 4>(op, B, na, g, I, p0, cnt);
