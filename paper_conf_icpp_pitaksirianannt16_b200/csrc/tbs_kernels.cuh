@@ -297,6 +297,22 @@ constexpr int kGuard = 32;
 
 extern __shared__ __align__(128) unsigned char tbs_smem[];  // dynamic smem; histogram at offset 0
 
+// Histogram increment. TBS_BOUNDS_CHECK (debug builds: compute-sanitizer is not available on the
+// GPU pool) traps if the address computed by the bucket / LEA.HI arithmetic leaves the histogram
+// words of the dynamic shared memory (replicas, guard rows, trash row).
+__device__ __forceinline__ void hist_inc(uint32_t a, long long hist_bytes) {
+#ifdef TBS_BOUNDS_CHECK
+  const uint32_t base = smem_addr(tbs_smem);
+  if (a < base || (long long)(a - base) + 4 > hist_bytes || (a & 3u) != 0u) {
+    printf("tbs bounds: smem increment at offset %lld outside [0, %lld) (block %d thread %d)\n",
+           (long long)a - (long long)base, hist_bytes, (int)blockIdx.x, (int)threadIdx.x);
+    __trap();
+  }
+#endif
+  (void)hist_bytes;
+  red_smem_inc(a);
+}
+
 // RANGED: bucket-range pass for nb beyond one shared-memory copy: only buckets
 // [klo, klo + rows) are counted in this launch (one predicated ATOMS); the host runs
 // ceil(nb / rows) passes over the triangle instead of falling back to global atomics.
@@ -437,8 +453,8 @@ struct SdhSmemOp {
     uint32_t ad0, ad1;
     bool in0 = true, in1 = true;
     float_addr2<V>(sqrt_sw2(s), ad0, ad1, in0, in1);
-    red_smem_inc(ad0);
-    red_smem_inc(ad1);
+    hist_inc(ad0, smem_bytes());
+    hist_inc(ad1, smem_bytes());
   }
 
   template <bool MASKED, int V>
@@ -492,11 +508,11 @@ struct SdhSmemOp {
       // address stays inside the allocation.
       const uint32_t trash = smem_addr(tbs_smem) + (uint32_t)(((rows << LOG2R) + (threadIdx.x & (R - 1))) * 4);
       const bool c0 = in0 && (!MASKED || pv > a0), c1 = in1 && (!MASKED || pv > a1);
-      red_smem_inc(c0 ? ad0 : trash);
-      red_smem_inc(c1 ? ad1 : trash);
+      hist_inc(c0 ? ad0 : trash, smem_bytes());
+      hist_inc(c1 ? ad1 : trash, smem_bytes());
     } else {
-      red_smem_inc(ad0);
-      red_smem_inc(ad1);
+      hist_inc(ad0, smem_bytes());
+      hist_inc(ad1, smem_bytes());
     }
   }
 
@@ -522,6 +538,9 @@ struct SdhSmemOp {
       }
       if (v != 0ull) {
         const int kk = k + (RANGED ? klo : 0);
+#ifdef TBS_BOUNDS_CHECK
+        if (kk < 0) { printf("tbs bounds: flush bucket %d < 0\n", kk); __trap(); }
+#endif
         out->add(kk < nb ? kk : nb - 1, v);
       }
     }
