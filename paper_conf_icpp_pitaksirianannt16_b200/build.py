@@ -20,7 +20,9 @@ def build(force=False, verbose=False, out=None, defines=()):
     if not force and os.path.exists(target) and all(os.path.getmtime(target) >= os.path.getmtime(d) for d in DEPS):
         return target
     tmp = target + f".tmp{os.getpid()}"
-    cmd = [NVCC] + FLAGS + [f"-D{d}" for d in defines] + ["-I", os.path.join(ROOT, "include"), "-o", tmp] + SRCS
+    extra = [d[len("NVCC:"):] for d in defines if d.startswith("NVCC:")]   # A/B builds: raw nvcc flags
+    defs = [f"-D{d}" for d in defines if not d.startswith("NVCC:")]
+    cmd = [NVCC] + FLAGS + extra + defs + ["-I", os.path.join(ROOT, "include"), "-o", tmp] + SRCS
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
