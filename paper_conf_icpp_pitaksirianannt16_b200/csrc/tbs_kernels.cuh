@@ -446,8 +446,9 @@ struct SdhSmemOp {
   // Float mode, unmasked pairs, square roots on the FMA pipe (the TBS_SW_SQRT slots).
   static constexpr bool kSwCapable = !LATTICE && !RANGED;
   // slot order of a partner group (run_chunk): anchor-major measured +1.0 % for float SDH at
-  // 1M, but -7.4 % for the lattice variants at 4M (profiles/r02_slot_order_ab.txt)
-  static constexpr bool kAnchorMajor = !LATTICE;
+  // 1M, but -7.4 % for the lattice variants at 4M and -20 % for bucket-range passes (65536
+  // buckets at 1M: 491 vs 409 ms; profiles/r02_slot_order_ab.txt, r02_ablations.jsonl)
+  static constexpr bool kAnchorMajor = !LATTICE && !RANGED;
   template <int V>
   __device__ __forceinline__ void pair2_sw(float2 s) {
     uint32_t ad0, ad1;
