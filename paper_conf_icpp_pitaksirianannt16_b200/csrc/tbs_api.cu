@@ -1097,6 +1097,67 @@ int staging(size_t bytes, void** out) {
   return TBS_OK;
 }
 
+// TBS_HOST_TRACE (diagnostics): per-phase host time of the small host-buffer path, averaged over
+// the calls and printed to stderr at exit.
+struct HostTrace {
+  static constexpr int kPhases = 8;
+  double ns[kPhases] = {0};
+  long long calls = 0;
+  std::chrono::steady_clock::time_point t;
+  bool on = getenv("TBS_HOST_TRACE") != nullptr;
+  void start() { if (on) t = std::chrono::steady_clock::now(); }
+  void mark(int k) {
+    if (!on) return;
+    const auto now = std::chrono::steady_clock::now();
+    ns[k] += std::chrono::duration<double, std::nano>(now - t).count();
+    t = now;
+  }
+  ~HostTrace() {
+    if (!on || !calls) return;
+    static const char* names[kPhases] = {"pointer_kind", "staging+memcpy", "host_dev_ptr", "malloc_async", "copy_kernel",
+                                         "op_call", "free_async", "poll"};
+    fprintf(stderr, "[tbs host trace] %lld calls, us per call:", calls);
+    for (int k = 0; k < kPhases; ++k) fprintf(stderr, " %s %.2f", names[k], ns[k] / calls * 1e-3);
+    fprintf(stderr, "\n");
+  }
+};
+HostTrace& host_trace() {
+  static HostTrace h;
+  return h;
+}
+
+// Per-thread device scratch of the small host-buffer path: [output | ticket], kept ZERO between
+// calls (zeroed once when allocated; afterwards the fused kernel's last CTA re-zeroes what the
+// call used, or the call itself on its fallback and error paths), so a call needs no allocation,
+// memset or copy kernel before its one launch.
+struct SmallScratch {
+  int dev = -1;
+  unsigned char* p = nullptr;
+  size_t bytes = 0;
+};
+int small_scratch(size_t bytes, unsigned char** out) {
+  static thread_local SmallScratch s;
+  int d = 0;
+  TBS_CUDA(cudaGetDevice(&d));
+  if (s.dev != d || s.bytes < bytes) {
+    const size_t want = std::max<size_t>(bytes, 65536 + 64);
+    unsigned char* p = nullptr;
+    TBS_CUDA(cudaMalloc((void**)&p, want));
+    TBS_CUDA(cudaMemset(p, 0, want));
+    // (a previous buffer of another device or smaller size is left allocated: calls are rare)
+    s = SmallScratch{d, p, want};
+  }
+  *out = s.p;
+  return TBS_OK;
+}
+// The points are pulled into device memory by a copy kernel first. TBS_SMALL_DIRECT=1 (A/B):
+// the fused kernel reads them from the mapped host buffer instead — measured slower (46 vs
+// 32.8 us per N = 4096 call: its 144 CTAs re-read the same lines over the host link).
+bool small_copy_in() {
+  static const bool v = [] { const char* e = getenv("TBS_SMALL_DIRECT"); return !(e && atoi(e) != 0); }();
+  return v;
+}
+
 // Run `fn(args_with_device_ptrs, dev_out)` for host or device buffers, synchronously.
 template <class Fn>
 int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_bytes, Fn fn,
@@ -1106,9 +1167,12 @@ int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_b
   if (!outp) return fail(TBS_EINVAL, "output is NULL");
   if (n >= 2 && !points) return fail(TBS_EINVAL, "points is NULL");
   int pk = 0, ok = 0;
+  HostTrace& tr = host_trace();
+  tr.start();
   int rc = pointer_kind(points, pk);
   if (!rc) rc = pointer_kind(outp, ok);
   if (rc) return rc;
+  tr.mark(0);
   if (points && (pk == 2) != (ok == 2)) return fail(TBS_EINVAL, "points and output must both be host or both device pointers");
   cudaStream_t st = cudaStreamPerThread;
   tbs_args a{};
@@ -1146,25 +1210,35 @@ int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_b
     }
     void* dst = pin_out ? static_cast<void*>(stage + pin_in) : outp;
     void *dsrc = nullptr, *ddst = nullptr;
+    tr.mark(1);
     if (cudaHostGetDevicePointer(&dsrc, const_cast<void*>(src), 0) == cudaSuccess &&
         cudaHostGetDevicePointer(&ddst, dst, 0) == cudaSuccess &&
         cudaHostGetDevicePointer(&dflag, const_cast<unsigned int*>(flag), 0) == cudaSuccess) {
-      const size_t dp_bytes = (pbytes + 255) / 256 * 256;
-      unsigned char* dbuf = nullptr;
-      cudaError_t e = cudaMallocAsync((void**)&dbuf, dp_bytes + out_bytes + 8, st);
-      if (e != cudaSuccess) return fail(TBS_ENOMEM, "cudaMallocAsync(%zu): %s", dp_bytes + out_bytes, cudaGetErrorString(e));
-      // [points | output | ticket]; the copy kernel also zeroes output + ticket, and the fused
-      // kernel's last CTA writes the result to the mapped host buffer (else a copy kernel does)
+      tr.mark(2);
+      // [output + ticket region (fixed, 64 KB + 64 B: zero on entry) | points (copy-in variant)]:
+      // the output and the ticket sit at the same place whatever the call's sizes, so the points
+      // of one call never land where a later call expects zeros
+      constexpr size_t kOutRegion = 65536 + 64;
+      const size_t dp_bytes = small_copy_in() ? (pbytes + 255) / 256 * 256 : 0;
+      unsigned char* dscr = nullptr;
+      if ((rc = small_scratch(kOutRegion + dp_bytes, &dscr))) return rc;
+      tr.mark(3);
       const int in_words = (int)(pbytes / 4), out_words = (int)(out_bytes / 4);
-      unsigned char* dout = dbuf + dp_bytes;
-      copy_in_zero<<<(in_words + 1023) / 1024 < 8 ? (in_words + 1023) / 1024 : 8, 1024, 0, st>>>(
-          reinterpret_cast<uint32_t*>(dbuf), static_cast<const uint32_t*>(dsrc), in_words,
-          reinterpret_cast<uint32_t*>(dout), out_words + 2);
-      g_launches.fetch_add(1);
-      a.points = reinterpret_cast<const float*>(dbuf);
+      unsigned char* dout = dscr;
+      unsigned char* dbuf = dscr + kOutRegion;
+      if (dp_bytes) {
+        copy_in_zero<<<(in_words + 1023) / 1024 < 8 ? (in_words + 1023) / 1024 : 8, 1024, 0, st>>>(
+            reinterpret_cast<uint32_t*>(dbuf), static_cast<const uint32_t*>(dsrc), in_words,
+            reinterpret_cast<uint32_t*>(dout), 0);
+        g_launches.fetch_add(1);
+      }
+      tr.mark(4);
+      // the fused kernel reads the points straight from the mapped page-locked host buffer
+      a.points = dp_bytes ? reinterpret_cast<const float*>(dbuf) : static_cast<const float*>(dsrc);
       SmallWriteBack& sw = small_wb();
       sw.wb.dst = static_cast<unsigned long long*>(ddst);
-      sw.wb.src = reinterpret_cast<const unsigned long long*>(dout);
+      sw.wb.src = reinterpret_cast<unsigned long long*>(dout);
+      sw.wb.rezero = 1;
       sw.wb.ticket = reinterpret_cast<unsigned int*>(dout + out_bytes);
       sw.wb.words = (int)(out_bytes / 8);
       static thread_local unsigned int seq = 0;
@@ -1175,13 +1249,15 @@ int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_b
       sw.active = true;
       sw.taken = false;
       rc = fn(&a, dout);
+      tr.mark(5);
       const bool taken = sw.taken;
       sw = SmallWriteBack{};
       if (!rc && !taken) {
         copy_words<<<1, 256, 0, st>>>(static_cast<uint32_t*>(ddst), reinterpret_cast<const uint32_t*>(dout), out_words);
         g_launches.fetch_add(1);
       }
-      cudaFreeAsync(dbuf, st);
+      if (rc || !taken) cudaMemsetAsync(dout, 0, out_bytes + 8, st);   // restore the zero scratch
+      tr.mark(6);
       bool done = false;
       if (!rc && taken) {
         // the kernel's last CTA signals completion through the mapped flag: poll it (a stream
@@ -1192,10 +1268,12 @@ int run_simple(const float* points, int64_t n, int dim, void* outp, size_t out_b
         }
       }
       if (!done) {
-        e = cudaStreamSynchronize(st);
+        const cudaError_t e = cudaStreamSynchronize(st);
         if (!rc && e != cudaSuccess) rc = fail(TBS_ECUDA, "sync: %s", cudaGetErrorString(e));
       }
       if (!rc && pin_out) memcpy(outp, dst, out_bytes);
+      tr.mark(7);
+      if (tr.on) tr.calls++;
       return rc;
     }
     cudaGetLastError();   // not mapped: the copy-engine path below

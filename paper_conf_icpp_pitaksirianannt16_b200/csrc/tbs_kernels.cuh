@@ -1032,13 +1032,16 @@ __global__ void push_peers(const unsigned long long* __restrict__ acc, int words
 // at `src` to mapped page-locked host memory `dst` (ticket zeroed before the launch).
 // Then it stores `seq` to the mapped host word `flag` (after a system fence), which the host
 // polls instead of waiting in a stream synchronisation.
+// rezero: the last CTA also zeroes `src` and the ticket after the write-back, so the caller's
+// cached scratch is zero again for its next call (no memset or copy kernel before the launch).
 struct WriteBack {
   unsigned long long* dst = nullptr;
-  const unsigned long long* src = nullptr;
+  unsigned long long* src = nullptr;
   unsigned int* ticket = nullptr;
   int words = 0;
   unsigned int* flag = nullptr;
   unsigned int seq = 0;
+  int rezero = 0;
 };
 
 template <class Op, int D, class C, int V>
@@ -1084,9 +1087,13 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel_small(const flo
     __syncthreads();
     if (s_last) {
       __threadfence();
-      for (int k = tid; k < wb.words; k += kThreads) wb.dst[k] = __ldcg(wb.src + k);
+      for (int k = tid; k < wb.words; k += kThreads) {
+        wb.dst[k] = __ldcg(wb.src + k);
+        if (wb.rezero) wb.src[k] = 0ull;
+      }
       __threadfence_system();
       __syncthreads();
+      if (tid == 0 && wb.rezero) *wb.ticket = 0u;   // every other CTA took its ticket before this one
       if (tid == 0 && wb.flag != nullptr) {
         *reinterpret_cast<volatile unsigned int*>(wb.flag) = wb.seq;
         __threadfence_system();

@@ -654,3 +654,26 @@ def test_host_small_path(tbs):
     h = tbs.sdh_host(pts[65536], w_of(nb), nb)                     # above the small-problem switch
     assert int(h.sum()) == 65536 * 65535 // 2
     assert h.tolist() == tbs.sdh(dev(pts[65536]), w_of(nb), nb).cpu().tolist()
+
+
+def test_host_small_path_mixed_sequence(tbs):
+    """The small host-buffer path keeps a per-thread device scratch zero between calls (the
+    fused kernel's last CTA re-zeroes what it used): interleave operations, point counts and
+    output sizes so every call's output region is one an earlier call dirtied differently."""
+    import ctypes
+    seq = [("sdh", 4096, 64), ("kde", 3000, 0), ("sdh", 2, 300), ("pcf", 16384, 0), ("sdh", 3000, 1000),
+           ("kde", 4096, 0), ("sdh", 16384, 8192), ("pcf", 5, 0), ("sdh", 4096, 64), ("kde", 2, 0)]
+    for rep in range(2):
+        for op, n, nb in seq:
+            p = g.uniform(n, 500 + n)
+            if op == "sdh":
+                ho, amb = oracle.sdh(p, w_of(nb), nb)
+                check_sdh_float(tbs.sdh_host(p, w_of(nb), nb), ho, amb)
+            elif op == "pcf":
+                co, ca = oracle.pcf(p, 0.05)
+                check_pcf_float(tbs.pcf_host(p, 0.05), co, ca)
+            else:
+                out = np.zeros(1, np.float64)
+                assert tbs.lib().tbs_kde(p.ctypes.data, n, ctypes.c_float(1.5), out.ctypes.data) == 0
+                ko = oracle.kde(p, 1.5)
+                assert abs(out[0] - ko) <= 1e-5 * max(ko, 1e-30)
