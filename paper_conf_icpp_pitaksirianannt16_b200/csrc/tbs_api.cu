@@ -264,6 +264,13 @@ SmallWriteBack& small_wb() {
   return w;
 }
 
+// TBS_SMALL_PDL=0 (A/B): launch the small fused kernel after the copy kernel without
+// programmatic dependent launch.
+bool small_pdl() {
+  static const bool v = [] { const char* e = getenv("TBS_SMALL_PDL"); return !(e && atoi(e) == 0); }();
+  return v;
+}
+
 template <class Op, int D, int V>
 int launch_small(const Device& dev, const tbs_args* a, const Op& op, cudaStream_t st, cudaEvent_t eb, cudaEvent_t ee,
                  const OutSink& sink) {
@@ -284,7 +291,23 @@ int launch_small(const Device& dev, const tbs_args* a, const Op& op, cudaStream_
     wb = small_wb().wb;
     small_wb().taken = true;
   }
-  kern<<<(unsigned)g.items, kThreads, (size_t)smem, st>>>(a->points, a->dim, g, op, sink, wb);
+  if (wb.dst != nullptr && small_pdl()) {
+    // after the host-buffer path's copy kernel: programmatic dependent launch (the grid starts
+    // early and waits in-kernel for the copy; griddepcontrol.wait)
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3((unsigned)g.items);
+    cfg.blockDim = dim3(kThreads);
+    cfg.dynamicSmemBytes = (size_t)smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    TBS_CUDA(cudaLaunchKernelEx(&cfg, kern, a->points, a->dim, g, op, sink, wb));
+  } else {
+    kern<<<(unsigned)g.items, kThreads, (size_t)smem, st>>>(a->points, a->dim, g, op, sink, wb);
+  }
   TBS_CUDA(cudaGetLastError());
   g_launches.fetch_add(1);
   if (ee) TBS_CUDA(cudaEventRecord(ee, st));

@@ -1057,6 +1057,10 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel_small(const flo
   int I, J;
   item_to_tile(g, (long long)blockIdx.x, I, J);
   const int p0 = J * C::TP;
+  // Programmatic dependent launch (host-buffer calls: this grid may start while the copy
+  // kernel that brings the points is still running): everything above overlaps it; wait for
+  // its completion before the first read of the points. A no-op without the launch attribute.
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   for (int p = tid; p < C::TP; p += kThreads) {
     const long long j = p0 + p;
 #pragma unroll
@@ -1106,6 +1110,7 @@ __global__ void __launch_bounds__(kThreads, C::MINB) pair_kernel_small(const flo
 // output words (+ the write-back ticket) the fused kernel accumulates into.
 __global__ void copy_in_zero(uint32_t* __restrict__ dst, const uint32_t* __restrict__ src, int words,
                              uint32_t* __restrict__ zero, int zero_words) {
+  asm volatile("griddepcontrol.launch_dependents;");   // the fused kernel may launch now (it waits)
   const int stride = gridDim.x * blockDim.x;
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < words; i += stride) dst[i] = src[i];
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < zero_words; i += stride) zero[i] = 0u;
