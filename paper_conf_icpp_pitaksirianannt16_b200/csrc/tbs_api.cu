@@ -60,6 +60,16 @@ static_assert(kMaxPeers == TBS_MAX_PEERS, "peer sink size");
 #ifndef TBS_PCF_MINB
 #define TBS_PCF_MINB 2
 #endif
+// kernel density (NEXT-2): 3 CTAs/SM measured +4.2 % over the 2PCF config (profiles/r02_sdh_config_ab.txt)
+#ifndef TBS_KDE_KA
+#define TBS_KDE_KA 8
+#endif
+#ifndef TBS_KDE_TP
+#define TBS_KDE_TP 1024
+#endif
+#ifndef TBS_KDE_MINB
+#define TBS_KDE_MINB 3
+#endif
 #ifndef TBS_LAT_KA
 #define TBS_LAT_KA 8
 #endif
@@ -86,6 +96,7 @@ static_assert(kMaxPeers == TBS_MAX_PEERS, "peer sink size");
 #define TBS_LAT_CFG TBS_LAT_KA, TBS_LAT_TP, TBS_LAT_MINB
 using SdhCfg = Cfg<TBS_SDH_CFG>;
 using PcfCfg = Cfg<TBS_PCF_CFG>;
+using KdeCfg = Cfg<TBS_KDE_KA, TBS_KDE_TP, TBS_KDE_MINB>;
 using LatCfg = Cfg<TBS_LAT_CFG>;
 using LatFastCfg = Cfg<TBS_LATF_CFG>;
 // Small problems (fewer work items than ~2 per SM with the main configs): finer tiles so
@@ -779,8 +790,8 @@ int kde_impl(const tbs_args* a, float gamma, double* sum) {
       rc = D == 3 ? launch_pair<KdeOp, 3, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee)
                   : launch_pair<KdeOp, 4, SmallCfg>(dev, soa, a, op, bbox, st, eb, ee);
     else
-      rc = D == 3 ? launch_pair<KdeOp, 3, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee)
-                  : launch_pair<KdeOp, 4, PcfCfg>(dev, soa, a, op, bbox, st, eb, ee);
+      rc = D == 3 ? launch_pair<KdeOp, 3, KdeCfg>(dev, soa, a, op, bbox, st, eb, ee)
+                  : launch_pair<KdeOp, 4, KdeCfg>(dev, soa, a, op, bbox, st, eb, ee);
   }
   release_soa(soa, st);
   return rc;
