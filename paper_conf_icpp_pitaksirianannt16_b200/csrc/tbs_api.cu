@@ -1013,6 +1013,9 @@ int hd_impl(const uint16_t* x, int64_t n, int d, int64_t rb, int64_t re, tbs_ker
 }
 
 // ---- NEXT-2: all-point kNN ---------------------------------------------------------------
+#ifndef TBS_KNN8_KA
+#define TBS_KNN8_KA 4   // anchors per thread for k <= 8 (A/B knob)
+#endif
 template <int K, int KA, int D>
 int knn_launch(const Device& dev, const tbs_args* a, const float* soa, int n_pad, int k, int32_t* idx, float* dist,
                cudaStream_t st) {
@@ -1072,11 +1075,11 @@ int knn_impl(const tbs_args* a, int k, int32_t* idx, float* dist) {
   rc = load_points(a, D, n_pad, &soa, nullptr, 0, st, &bbox, INFINITY);
   if (!rc) {
     if (D == 3) rc = k <= 4 ? knn_launch<4, 4, 3>(dev, a, soa, n_pad, k, idx, dist, st)
-                     : k <= 8 ? knn_launch<8, 4, 3>(dev, a, soa, n_pad, k, idx, dist, st)
+                     : k <= 8 ? knn_launch<8, TBS_KNN8_KA, 3>(dev, a, soa, n_pad, k, idx, dist, st)
                      : k <= 16 ? knn_launch<16, 2, 3>(dev, a, soa, n_pad, k, idx, dist, st)
                                : knn_launch<32, 2, 3>(dev, a, soa, n_pad, k, idx, dist, st);
     else rc = k <= 4 ? knn_launch<4, 4, 4>(dev, a, soa, n_pad, k, idx, dist, st)
-              : k <= 8 ? knn_launch<8, 4, 4>(dev, a, soa, n_pad, k, idx, dist, st)
+              : k <= 8 ? knn_launch<8, TBS_KNN8_KA, 4>(dev, a, soa, n_pad, k, idx, dist, st)
               : k <= 16 ? knn_launch<16, 2, 4>(dev, a, soa, n_pad, k, idx, dist, st)
                         : knn_launch<32, 2, 4>(dev, a, soa, n_pad, k, idx, dist, st);
   }

@@ -105,8 +105,11 @@ __device__ __forceinline__ void chunk(const float* __restrict__ B, int p0, const
 // Segment y: partner chunks [y * seg, min((y + 1) * seg, n_chunks)).
 // S == 1: writes the first kout entries (idx, sqrt(s)) of rows in [rb, re) directly;
 // else the K-list (s, j) to part_s/part_j [y][row - rb][K].
+#ifndef TBS_KNN_MINB16
+#define TBS_KNN_MINB16 2   // resident CTAs per SM for K <= 16 (A/B knob)
+#endif
 template <int K, int KA, int D>
-__global__ void __launch_bounds__(kThreads, K <= 16 ? 2 : 1) knn_kernel(const float* __restrict__ soa, int n, int n_pad, int rb, int re,
+__global__ void __launch_bounds__(kThreads, K <= 16 ? TBS_KNN_MINB16 : 1) knn_kernel(const float* __restrict__ soa, int n, int n_pad, int rb, int re,
                                                        int I0, int seg, int n_chunks, int kout,
                                                        float* __restrict__ part_s, int* __restrict__ part_j,
                                                        int* __restrict__ out_idx, float* __restrict__ out_dist) {
