@@ -104,6 +104,9 @@ using LatFastCfg = Cfg<TBS_LATF_CFG>;
 #ifndef TBS_SMALL_TP
 #define TBS_SMALL_TP 128
 #endif
+#ifndef TBS_SMALL_LOG2R
+#define TBS_SMALL_LOG2R 5   // histogram replicas (2^x) of the small fused kernel
+#endif
 #ifndef TBS_SMALL_KA
 #define TBS_SMALL_KA 2
 #endif
@@ -657,15 +660,17 @@ int sdh_impl(const tbs_args* a, float w, int nb, uint64_t* hist) {
   const int D = a->dim <= 3 ? 3 : 4;
   if (!lattice && !pl.global && pl.passes == 1 && pl.log2r == 5 && small_fused(dev, a)) {
     // small problem: zero the output, one fused launch (clamp variant: no bounding box)
-    SdhSmemOp<5, false> op{};
+    using SOp = SdhSmemOp<TBS_SMALL_LOG2R, false>;
+    SOp op{};
     op.nb = nb;
     op.rows = nb + kGuard;
     op.inv_w = (float)(1.0 / (double)w);
-    op.flush_every = (int)std::max<long long>(1, 0xffffffffll / ((long long)kWarps * SmallCfg::KA * SmallCfg::TP) - 1);
+    op.flush_every = (int)std::max<long long>(
+        1, 0xffffffffll / ((long long)(32 >> TBS_SMALL_LOG2R) * kWarps * SmallCfg::KA * SmallCfg::TP) - 1);
     if (!small_wb().active || peers) TBS_CUDA(cudaMemsetAsync(h, 0, (size_t)nb * 8, st));
     cudaEvent_t eb = (cudaEvent_t)a->ev_begin, ee = (cudaEvent_t)a->ev_end;
-    rc = D == 3 ? launch_small<SdhSmemOp<5, false>, 3, 1>(dev, a, op, st, eb, ee, sink)
-                : launch_small<SdhSmemOp<5, false>, 4, 1>(dev, a, op, st, eb, ee, sink);
+    rc = D == 3 ? launch_small<SOp, 3, 1>(dev, a, op, st, eb, ee, sink)
+                : launch_small<SOp, 4, 1>(dev, a, op, st, eb, ee, sink);
     if (!rc && peers) rc = push_to_peers(a, acc, nb, st);
     if (acc) cudaFreeAsync(acc, st);
     return rc;
