@@ -1178,15 +1178,18 @@ struct SmallScratch {
   size_t bytes = 0;
 };
 int small_scratch(size_t bytes, unsigned char** out) {
-  static thread_local SmallScratch s;
+  constexpr int kDevs = 16;
+  static thread_local SmallScratch per_dev[kDevs];   // one buffer per device and thread
   int d = 0;
   TBS_CUDA(cudaGetDevice(&d));
-  if (s.dev != d || s.bytes < bytes) {
-    const size_t want = std::max<size_t>(bytes, 65536 + 64);
+  if (d < 0 || d >= kDevs) return fail(TBS_EUNSUPPORTED, "small host path: device %d >= %d", d, kDevs);
+  SmallScratch& s = per_dev[d];
+  if (s.bytes < bytes) {
+    const size_t want = std::max<size_t>(bytes, 65536 + 64 + 16384 * 16);   // output region + the largest points
     unsigned char* p = nullptr;
     TBS_CUDA(cudaMalloc((void**)&p, want));
     TBS_CUDA(cudaMemset(p, 0, want));
-    // (a previous buffer of another device or smaller size is left allocated: calls are rare)
+    if (s.p) cudaFree(s.p);   // (synchronous; the previous call on this thread has completed)
     s = SmallScratch{d, p, want};
   }
   *out = s.p;
