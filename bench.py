@@ -55,6 +55,7 @@ WORKLOADS = {
     "pairmatrix_hd_64k_d64": ("pairmatrix_hd", "uniform", 1 << 16, 7, dict(d=64, gamma=1.0 / 64)),  # NEXT-3
     "knn_uniform_1m_k8": ("knn", "uniform", 1 << 20, 2, dict(k=8)),  # NEXT-2 (all-point kNN)
     "pairmatrix_hd_64k_d512": ("pairmatrix_hd", "uniform", 1 << 16, 7, dict(d=512, gamma=1.0 / 512)),
+    "rdf_uniform_1m": ("rdf", "uniform", 1 << 20, 2, dict(nb=256, volume=1.0)),  # NEXT-1 (SDH + normalisation)
 }
 METRIC = "SDH pair-distances/sec (G pairs/s) at N=1M–4M, 1/2/4/8 B200, % of roofline"
 
@@ -168,6 +169,8 @@ def oracle_rate(op, p, params, rows):
     t0 = time.perf_counter()
     if op == "sdh":
         oracle.sdh(p, float(np.float32(math.sqrt(3) / params["nb"])), params["nb"], rows=rows)
+    elif op == "rdf":
+        oracle.rdf_points(p, float(np.float32(math.sqrt(3) / params["nb"])), params["nb"], params["volume"], rows=rows)
     elif op == "sdh_lattice":
         oracle.sdh_lattice(p, 1, 0, params["nb"], rows=rows)
     elif op == "pcf":
@@ -338,10 +341,12 @@ def main():
     st = torch.cuda.current_stream(dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     nb = params.get("nb", 1)
-    w = float(np.float32(math.sqrt(3) / nb)) if op == "sdh" else params.get("w", 1.0)
+    w = float(np.float32(math.sqrt(3) / nb)) if op in ("sdh", "rdf") else params.get("w", 1.0)
     out = None
     if op in ("sdh", "sdh_lattice"):
         out = torch.empty(nb, dtype=torch.int64, device=dev)
+    elif op == "rdf":
+        out = torch.empty(nb, dtype=torch.float64, device=dev)
     elif op == "pcf":
         out = torch.empty(1, dtype=torch.int64, device=dev)
     elif op == "kde":
@@ -375,6 +380,8 @@ def main():
             tbs.sdh(pts, w, nb, out=out, events=events, group=pg, sink=sink)
         elif op == "sdh_lattice":
             tbs.sdh(pts, w, nb, lattice=True, out=out, events=events, group=pg, sink=sink)
+        elif op == "rdf":
+            tbs.rdf(pts, w, nb, params["volume"], out=out, events=events, group=pg)
         elif op == "pcf":
             tbs.pcf(pts, params["r"], out=out, events=events, group=pg, sink=sink)
         elif op == "kde":
@@ -513,7 +520,7 @@ def main():
                 "frac": pairs_s / peak, "peak_source": f"{bound_note}; 148 SMs x unit lanes/clk x "
                                                       f"{pk['f_max'] / 1e6:.0f} MHz (DESIGN.md §Roofline)",
                 "frac_fp32": pairs_s * 6 / pk["fp32"]}
-        if op in ("sdh", "sdh_lattice"):
+        if op in ("sdh", "sdh_lattice", "rdf"):
             roof["mufu_cap"] = pk["mufu"] / 1e9         # one MUFU.SQRT per pair: this design's ceiling
             roof["frac_of_mufu_cap"] = pairs_s / pk["mufu"]
             if nb + 32 > 768:
@@ -540,11 +547,12 @@ def main():
 
     # e2e: host buffers through the public API, H2D of the points and D2H of the result each step
     e2e = None
-    if op in ("sdh", "sdh_lattice", "pcf", "kde", "knn"):
+    if op in ("sdh", "sdh_lattice", "pcf", "kde", "knn", "rdf"):
         ph = torch.from_numpy(p_host).pin_memory()
         if world == 1 and op != "sdh_lattice":     # the simple host-pointer entry points
             hh = np.zeros(nb if op == "sdh" else 1, np.uint64)
             kh = np.zeros(1, np.float64)
+            gh = np.zeros(nb, np.float64)
 
             # the C-ABI host-buffer entry points (tbs_sdh / tbs_pcf / tbs_kde: the north star's
             # signatures) called directly, arguments marshalled once; status checked every call
@@ -555,6 +563,8 @@ def main():
             def e2e_step():
                 if op == "sdh":
                     rc = L.tbs_sdh(pptr, n, 3, cw, nb, hh.ctypes.data)
+                elif op == "rdf":
+                    rc = L.tbs_rdf(pptr, n, 3, cw, nb, ctypes.c_double(params["volume"]), gh.ctypes.data)
                 elif op == "kde":
                     rc = L.tbs_kde(pptr, n, cg, kh.ctypes.data)
                 elif op == "knn":
@@ -571,6 +581,8 @@ def main():
                 d = ph.to(dev, non_blocking=True)
                 if op == "sdh":
                     r = tbs.sdh(d, w, nb, group=pg, sink=sink)
+                elif op == "rdf":
+                    r = tbs.rdf(d, w, nb, params["volume"], group=pg)
                 elif op == "sdh_lattice":
                     r = tbs.sdh(d, w, nb, lattice=True, group=pg, sink=sink)
                 elif op == "kde":
@@ -610,8 +622,10 @@ def main():
                "parallelism": f"rows{world}" if world > 1 else "single",
                "step": "loader + pair kernel + flush" + (f" + combine ({combine})" if world > 1 else ""),
                "combine": combine, "cuda_graph": graph is not None}
-        if op == "sdh":
+        if op in ("sdh", "rdf"):
             cfg["bucket_width"] = w
+        if op == "rdf":
+            cfg["step"] += " + RDF normalisation kernel (an nb + 1-bucket SDH)"
         line = {"metric": METRIC if op in ("sdh", "sdh_lattice") else f"{op} throughput ({unit})",
                 "value": value, "unit": unit, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
                 "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "strong",
