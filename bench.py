@@ -235,7 +235,8 @@ def run_reference(args, wl):
         tot_u += u
         tot_t += dt
     v = tot_u / tot_t / 1e9
-    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": unit, "n_gpus": args.gpus,
+    metric = METRIC if op in ("sdh", "sdh_lattice") else f"{op} throughput ({unit})"   # as the tbs arm names it
+    line = {"impl": "reference", "metric": metric, "value": v, "unit": unit, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_t / args.steps * 1e3,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": wl, "n": n, "distribution": dist_, "seed": seed, **params},
