@@ -153,8 +153,9 @@ class PeerSink:
     """Buffers of the fused combine (TBS_OUT_PEERS): one int64[words] device buffer per rank
     of `group`, each mapped into every rank (CUDA IPC; over NVLink between GPUs; every peer
     must be reachable with native atomics). A call with ``sink=`` accumulates its row strip's
-    partial locally and its last kernel adds it into all of them (system-scope atomics: words x
-    ranks remote adds per rank), so after ``finish()`` each rank's buffer holds the all-reduced
+    partial locally and the pair kernel's last CTA adds it into all of them (system-scope
+    atomics: words x ranks remote adds per rank; after multi-launch output stages, one extra
+    kernel does), so after ``finish()`` each rank's buffer holds the all-reduced
     result — the collective is fused into the call instead of a separate NCCL all_reduce.
 
     Every rank holds two buffers (parity p = result index & 1), so one host barrier per
@@ -325,7 +326,8 @@ def sdh(points, bucket_width: float, nbuckets: int, *, rows=None, lattice: bool 
     exact integer bucketing (integer-valued points, bucket_width = m * 2^-j).
     group: a torch.distributed process group: each rank computes its pair-balanced
     strip (rank_rows) and the partial histograms are summed with one all_reduce, or, with
-    sink=PeerSink(nbuckets, group), by the kernels' own flush into every rank's buffer.
+    sink=PeerSink(nbuckets, group), by the pair kernel itself (its last CTA adds the rank's partial
+    into every rank's buffer over peer memory).
     validate=True: TBS_VALIDATE (debug; raises on non-finite coordinates and, with lattice, on a
     violated exact-lattice contract).
     """
