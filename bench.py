@@ -49,6 +49,7 @@ WORKLOADS = {
     "sdh_uniform_4m": ("sdh", "uniform", 1 << 22, 6, dict(nb=256)),         # north-star target line
     "sdh_uniform_2m_16k": ("sdh", "uniform", 1 << 21, 4, dict(nb=16384)),   # configs[3]
     "sdh_lattice_4m": ("sdh_lattice", "lattice", 160 ** 3, 6, dict(nb=256, w=1.0)),
+    "sdh_lattice_2m_16k": ("sdh_lattice", "lattice", 128 ** 3, 4, dict(nb=16384, w=2.0 ** -6)),  # configs[3], exact mode
     "pcf_clustered_4m": ("pcf", "clustered", 1 << 22, 3, dict(r=0.03)),     # configs[2]
     "pairmatrix_64k": ("pairmatrix", "uniform", 1 << 16, 5, dict(gamma=1.0)),  # configs[4]
     "kde_uniform_1m": ("kde", "uniform", 1 << 20, 2, dict(gamma=1.0)),        # NEXT-2 (Type-I float sum)

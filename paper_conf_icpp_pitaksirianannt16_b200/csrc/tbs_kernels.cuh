@@ -367,11 +367,17 @@ struct SdhSmemOp {
       const double X = (floor(xmax) + 1.0) * (double)m;
       if (!RANGED && smax < 16777216.0 && X * X < 131072.0 && xmax * (1.0 + 1.0 / 262144.0) + 2.0 < (double)(nb + kGuard))
         return 4;
-      if (smax < 8388608.0 && S < 16777216.0 && e * e < 16777216.0) {
-        // fast variant: estimate k0 <= floor(sqrt(S) / m * (1 + 2^-16)) must stay a valid row
-        if (!RANGED && sqrt(S) / (double)m * (1.0 + 1.0 / 32768.0) + 2.0 < (double)(nb + kGuard)) return 0;
-        return 1;
-      }
+      // One-sided fp32 variant 0 (pair2, V == 0). It needs: s exact in fp32 (smax < 2^23);
+      // k0 = floor(q c_up) in {k, k + 1}, i.e. x (1 + 2^-16) < k + 2 for every reachable
+      // x = sqrt(4^j s) / m (x < 2^15 leaves a 2x margin); e0 = k0 m 2^-j exact (k0 m < 2^24);
+      // the sign of t = s - e0^2 exact — one FFMA: the product is exact inside it and a rounding
+      // never flips a sign, s and e0^2 being multiples of 4^-j far above the underflow range —
+      // and every estimate a valid row (no clamp). It does NOT need 4^j s < 2^24 (r02: the C4
+      // lattice, w = 2^-6, X up to 14080, took the 32-bit integer variant for that reason).
+      if (!RANGED && smax < 8388608.0 && xmax < 32768.0 && (kmax + 1.0) * (double)m < 16777216.0 &&
+          xmax * (1.0 + 1.0 / 32768.0) + 2.0 < (double)(nb + kGuard))
+        return 0;
+      if (smax < 8388608.0 && S < 16777216.0 && e * e < 16777216.0) return 1;
       const double em = (double)(nb + 1) * (double)m;
       if (smax < 8388608.0 && S < 4294967296.0 && em * em < 4294967296.0) return 2;
       return 3;
@@ -466,7 +472,7 @@ struct SdhSmemOp {
       float_addr2<V>(make_float2(sqrt_approx(s.x), sqrt_approx(s.y)), ad0, ad1, in0, in1);
     } else if (V == 0) {
       // Lattice, fast variant. The estimate uses a scale rounded UP by 2^-17, far above the
-      // sqrt.approx + rounding error (~2^-22) and far below 1/x (x = sqrt(4^j s)/m < 4096),
+      // sqrt.approx + rounding error (~2^-22) and far below 1/x (x = sqrt(4^j s)/m < 2^15),
       // so k0 = floor(estimate) is k or k + 1, never less. One exact check decides:
       //   e0 = k0 m 2^-j  (one FFMA: (2^23 + k0) mj - 2^23 mj, exact as k0 m < 2^24)
       //   t  = s - e0^2   (one FFMA; its sign is exact: -0 never arises, t = 0 is a tie -> k0)

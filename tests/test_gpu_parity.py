@@ -164,6 +164,19 @@ def test_sdh_lattice_bias_only_boundary(tbs):
     assert h.tolist() == oracle.sdh_lattice(p, 1, 0, 400).tolist()
 
 
+@pytest.mark.parametrize("L,j", [(20, 9), (17, 10)])
+def test_sdh_lattice_one_sided_large_x(tbs, L, j):
+    """One-sided fp32 exact variant where 4^j s exceeds 2^24 (the r02 relaxation): w = 2^-j on
+    {0..L-1}^3, x = sqrt(4^j s) reaches ~16900 (L 20, j 9) and ~28400 (L 17, j 10) — up to
+    0.87 of its 2^15 admission limit; corners added so the extreme distances occur."""
+    p = g.lattice(L, 22 + j)[:6000]
+    c = float(L - 1)
+    p = np.concatenate([p, np.array([[0, 0, 0], [c, c, c], [c, 0, 0], [0, c, c]], np.float32)])
+    nb = int(math.ceil(math.sqrt(3.0) * c * 2 ** j)) + 40
+    h = sdh_gpu(tbs, p, 2.0 ** -j, nb, lattice=True)
+    assert h.tolist() == oracle.sdh_lattice(p, 1, j, nb).tolist()
+
+
 def test_sqrt_approx_bound():
     """The bias-only lattice variant assumes |sqrt.approx(s) / sqrt(s) - 1| <= 2^-22 for every
     integer s < 2^24 (exhaustive on this GPU; tools/sqrt_bound.cu), with its 2^-19 bias
