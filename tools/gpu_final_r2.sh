@@ -12,7 +12,7 @@ python bench.py > $O/bench_default.json 2> $O/bench_default.err
 timeout 900 python bench.py --impl reference --steps 2 --warmup 3 > $O/bench_reference.json 2> $O/bench_reference.err
 B="timeout 900 python bench.py --no-cpu-baseline"
 for wl in sdh_uniform_4m sdh_clustered_1m sdh_uniform_2m_16k sdh_lattice_4m sdh_uniform_4k pcf_clustered_4m pairmatrix_64k kde_uniform_1m knn_uniform_1m_k8 pairmatrix_hd_64k_d64 pairmatrix_hd_64k_d512; do
-  S=10; case $wl in sdh_uniform_4m|sdh_lattice_4m|pcf_clustered_4m|sdh_uniform_2m_16k) S=3;; sdh_uniform_4k) S=50;; esac
+  S=10; case $wl in sdh_uniform_4m|sdh_lattice_4m|pcf_clustered_4m|sdh_uniform_2m_16k) S=3;; sdh_uniform_4k) S=3000;; esac
   $B --workload $wl --steps $S > $O/bench_$wl.json 2> $O/bench_$wl.err
 done
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_sdh_uniform_1m.csv \
